@@ -1,0 +1,152 @@
+// Shared constants, data structures and block/warp primitives of the AC-SpGEMM
+// CUDA path (sm_100a).  Nothing here is shared with oracle/ (the test oracle).
+//
+// Tile constants (§4: "sorts 8 elements per thread and keeps up
+// to 4 elements per thread"; "256/512 non-zeros" per block for global load
+// balancing).  They are fixed per build: they decide the summation tree and hence
+// the bits of every result (reading R7 in DESIGN.md).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace acs {
+
+constexpr int THREADS = 256;                 // threads per CTA (L344)
+constexpr int ITEMS = 8;                     // sorted elements per thread (L556)
+constexpr int CAP = THREADS * ITEMS;         // products per local ESC iteration
+constexpr int IDXBITS = 11;                  // log2(CAP): position bits in a sort word
+constexpr int NNZ_PER_THREAD = 2;            // A entries per thread (L344)
+constexpr int NPB = THREADS * NNZ_PER_THREAD;// NNZ_PER_BLOCK (Alg. 1, Alg. 2)
+constexpr int KEEP = 4 * THREADS;            // max kept elements of the last row (L556)
+constexpr int RADIX_BITS = 5;                // digit width of one radix-sort pass
+constexpr int DEFAULT_SEGMENTS = 8;          // canonical segments
+constexpr int MAX_SEGMENTS = 64;
+constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)
+static_assert((1 << IDXBITS) == CAP, "IDXBITS must be log2(CAP)");
+static_assert(KEEP <= CAP / 2, "kept row must leave room for new products");
+
+// A chunk of C (§3.2.4: "each chunk holds its starting row, element
+// count and number of elements in the first and last row"; the chunk id (block,
+// running number) gives the global order, L430).  Column indices and values live in
+// the pool arrays at [data_off, data_off + count).
+struct ChunkDesc {
+  int64_t data_off;
+  int32_t first_row, last_row;
+  int32_t count, first_count, last_count;
+  int32_t flags;          // bit0: first row shared, bit1: last row shared (set by MCC)
+};
+static_assert(sizeof(ChunkDesc) == 32, "ChunkDesc layout");
+
+// A row of C that spans >= 2 chunks (the "shared rows" array, L432).
+struct SharedRow {
+  int32_t row;
+  int32_t first_chunk;    // dense global chunk index of the first chunk holding the row
+  int32_t nchunks;
+  int32_t total;          // sum of the row's element counts over its chunks (pre-merge)
+  int64_t merge_off;      // where the merged row goes in the merge pool
+  int32_t merged;         // merged element count (written by the merge kernels)
+  int32_t kind;           // 0 multi, 1 path, 2 search
+};
+
+// ---------------------------------------------------------------- helpers --
+
+__device__ __forceinline__ int bit_width_u64(uint64_t x) { return x ? 64 - __clzll((long long)x) : 0; }
+
+template <typename T> struct ValueTraits;
+template <> struct ValueTraits<float> { static constexpr int bytes = 4; };
+template <> struct ValueTraits<double> { static constexpr int bytes = 8; };
+
+__device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+// Block-wide exclusive prefix sum of one value per thread (fixed shuffle tree).
+// `scratch` needs THREADS/32 + 1 elements.  Returns the exclusive prefix; *total
+// receives the block sum.  Contains two __syncthreads().
+template <typename V>
+__device__ __forceinline__ V block_exclusive_sum(V x, V* scratch, V* total) {
+  const int lane = lane_id(), w = warp_id();
+  V inc = x;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    V y = __shfl_up_sync(0xffffffffu, inc, d);
+    if (lane >= d) inc += y;
+  }
+  if (lane == 31) scratch[w] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    V run = 0;
+    for (int i = 0; i < THREADS / 32; ++i) { V t = scratch[i]; scratch[i] = run; run += t; }
+    scratch[THREADS / 32] = run;
+  }
+  __syncthreads();
+  V res = scratch[w] + inc - x;
+  *total = scratch[THREADS / 32];
+  __syncthreads();          // scratch may be reused by the caller right away
+  return res;
+}
+
+// Block-wide inclusive max scan (one value per thread).  Two __syncthreads().
+__device__ __forceinline__ int block_inclusive_max(int x, int* scratch) {
+  const int lane = lane_id(), w = warp_id();
+  int inc = x;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    int y = __shfl_up_sync(0xffffffffu, inc, d);
+    if (lane >= d) inc = max(inc, y);
+  }
+  if (lane == 31) scratch[w] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int run = 0;
+    for (int i = 0; i < THREADS / 32; ++i) { int t = scratch[i]; scratch[i] = run; run = max(run, t); }
+  }
+  __syncthreads();
+  int res = max(scratch[w], inc);
+  __syncthreads();
+  return res;
+}
+
+// Block-wide exclusive max scan (identity 0, the "clear(Offsets)" value of Alg. 2).
+__device__ __forceinline__ int block_exclusive_max(int x, int* scratch) {
+  const int lane = lane_id(), w = warp_id();
+  int inc = x;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    int y = __shfl_up_sync(0xffffffffu, inc, d);
+    if (lane >= d) inc = max(inc, y);
+  }
+  int ex = __shfl_up_sync(0xffffffffu, inc, 1);
+  if (lane == 0) ex = 0;
+  if (lane == 31) scratch[w] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int run = 0;
+    for (int i = 0; i < THREADS / 32; ++i) { int t = scratch[i]; scratch[i] = run; run = max(run, t); }
+  }
+  __syncthreads();
+  int res = max(scratch[w], ex);
+  __syncthreads();
+  return res;
+}
+
+// Block-wide min/max reduction of four ints (rmin, rmax, cmin, cmax).
+__device__ __forceinline__ void block_minmax4(int& a_min, int& a_max, int& b_min, int& b_max, int* scratch) {
+  a_min = __reduce_min_sync(0xffffffffu, a_min);
+  a_max = __reduce_max_sync(0xffffffffu, a_max);
+  b_min = __reduce_min_sync(0xffffffffu, b_min);
+  b_max = __reduce_max_sync(0xffffffffu, b_max);
+  const int w = warp_id();
+  if (lane_id() == 0) {
+    scratch[4 * w + 0] = a_min; scratch[4 * w + 1] = a_max;
+    scratch[4 * w + 2] = b_min; scratch[4 * w + 3] = b_max;
+  }
+  __syncthreads();
+  a_min = scratch[0]; a_max = scratch[1]; b_min = scratch[2]; b_max = scratch[3];
+  for (int i = 1; i < THREADS / 32; ++i) {
+    a_min = min(a_min, scratch[4 * i + 0]); a_max = max(a_max, scratch[4 * i + 1]);
+    b_min = min(b_min, scratch[4 * i + 2]); b_max = max(b_max, scratch[4 * i + 3]);
+  }
+  __syncthreads();
+}
+
+}  // namespace acs

@@ -1,0 +1,289 @@
+// Stage 2 — Adaptive chunk-based ESC (§3.2).
+//
+// One CTA per block of NPB nonzeros of A.  Per CTA:
+//   Fetch A (§3.2.1): coalesced load of the block's A entries, B row starts and
+//     lengths, and a dense local row dictionary (local id = rank of the row among the
+//     block's rows; its bit width is bounded by log2(NPB) like the paper's dictionary).
+//   placework (Alg. 2), then iterate:
+//     receivework(CAP - kept) -> expand (§3.2.3) -> radix sort of
+//     (row, col) keys with the bit range reduced to the rows and columns present
+//     (L342-L344) -> compaction scan (Alg. 3) -> completed rows go to a chunk, the
+//     last row is kept in shared memory when it is not yet complete and has at most
+//     KEEP elements (L364-L366) -> per-row counts (L362).
+// Chunk allocation is deterministic (reading R8): block b writes its chunks to a
+// slot range sized from its exact product count (stage 1), so no atomics, no
+// restarts, and the chunk id (block, running number) is the global order (L430).
+#include <climits>
+#include "esc_core.cuh"
+#include "kernels.cuh"
+
+namespace acs {
+
+template <typename T>
+struct EscSmem {
+  SortSmem<T> s;
+  T a_val[NPB];
+  int a_bstart[NPB];
+  int a_lrow[NPB];
+  int row_of[NPB];
+  int wd[NPB + 1];
+  int rp_cache[THREADS + 1];
+  int kept_col[KEEP];
+  T kept_val[KEEP];
+};
+
+struct EscState {
+  int kept, kept_lrow, kept_cmin, kept_cmax;
+  int seq;
+  int64_t wofs;
+};
+
+// One local ESC iteration after expansion: build words, sort, compact, emit.
+template <typename Word, typename T>
+__device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, EscState& st, int consume,
+                                              int size_after, const int (&ares)[ITEMS], const int (&lr)[ITEMS],
+                                              const int (&col)[ITEMS], const T (&v)[ITEMS], int rmin, int cmin,
+                                              int rowbits, int colbits, int64_t pool_base, int64_t desc_base) {
+  const int tid = threadIdx.x;
+  const int kept = st.kept;
+  const int n = kept + consume;
+  Word* sw = reinterpret_cast<Word*>(S.s.words);
+  // positions: kept elements first (they sort before equal keys, L366), then product c
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    if (ares[i] >= 0) {
+      const int pos = kept + i * THREADS + tid;
+      const Word key = ((Word)(lr[i] - rmin) << colbits) | (Word)(col[i] - cmin);
+      sw[pos] = (key << IDXBITS) | (Word)pos;
+      S.s.vals[pos] = v[i];
+    }
+  }
+  for (int p = tid; p < kept; p += THREADS) {
+    const Word key = ((Word)(st.kept_lrow - rmin) << colbits) | (Word)(S.kept_col[p] - cmin);
+    sw[p] = (key << IDXBITS) | (Word)p;
+    S.s.vals[p] = S.kept_val[p];
+  }
+  for (int p = n + tid; p < CAP; p += THREADS) sw[p] = ~(Word)0;
+  __syncthreads();
+
+  CElem<Word, T> x[ITEMS];
+  sort_and_scan<Word, T>(S.s, n, rowbits + colbits, colbits, x);
+
+  int* misc = S.s.misc;
+  if (tid == (n - 1) / ITEMS) {
+    const int i = (n - 1) % ITEMS;
+#pragma unroll
+    for (int q = 0; q < ITEMS; ++q) {
+      if (q == i) {
+        misc[0] = st_count(x[q].state);
+        misc[1] = st_row_count(x[q].state);
+        misc[2] = (int)(x[q].key >> colbits);
+      }
+    }
+  }
+  __syncthreads();
+  const int total = misc[0], rc_last = misc[1], lastrel = misc[2];
+  // keep the last row for the next iteration (L366) unless the block is done or the
+  // row no longer fits the kept budget (reading R13: then it is written as a partial
+  // chunk and merged later)
+  const bool keep = size_after > 0 && rc_last <= KEEP;
+  const int nchunk = total - (keep ? rc_last : 0);
+  int* stage_col = reinterpret_cast<int*>(S.s.words);
+  T* stage_val = S.s.vals;
+  const Word colmask = colbits ? (((Word)1 << colbits) - (Word)1) : (Word)0;
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    const uint32_t s = x[i].state;
+    if (s & 1u) {
+      const int p = st_count(s) - 1;
+      const int c = cmin + (int)(x[i].key & colmask);
+      const int rel = (int)(x[i].key >> colbits);
+      if (p < nchunk) {
+        stage_col[p] = c;
+        stage_val[p] = x[i].val;
+        if (st_row_end(s)) {
+          const int rc = st_row_count(s);
+          a.row_count[S.row_of[rmin + rel]] = rc;        // per-row counter (L362)
+          if (rel == 0) misc[3] = rc;
+          if (p == nchunk - 1) { misc[4] = rel; misc[5] = rc; }
+        }
+      } else {
+        S.kept_col[p - nchunk] = c;
+        S.kept_val[p - nchunk] = x[i].val;
+      }
+    }
+  }
+  __syncthreads();
+  if (nchunk > 0) {
+    // chunk write through shared memory for coalescing (L424-L426)
+    const int64_t dst = pool_base + st.wofs;
+    T* pv = reinterpret_cast<T*>(a.pool_val);
+    for (int p = tid; p < nchunk; p += THREADS) {
+      a.pool_col[dst + p] = stage_col[p];
+      pv[dst + p] = stage_val[p];
+    }
+    if (tid == 0) {
+      ChunkDesc d;
+      d.data_off = dst;
+      d.first_row = S.row_of[rmin];
+      d.last_row = S.row_of[rmin + misc[4]];
+      d.count = nchunk;
+      d.first_count = misc[3];
+      d.last_count = misc[5];
+      d.flags = 0;
+      a.descs[desc_base + st.seq] = d;
+    }
+    st.seq += 1;
+    st.wofs += nchunk;
+  }
+  st.kept = keep ? rc_last : 0;
+  if (keep) {
+    st.kept_lrow = rmin + lastrel;
+    st.kept_cmin = S.kept_col[0];
+    st.kept_cmax = S.kept_col[st.kept - 1];
+  }
+  __syncthreads();
+}
+
+template <typename T>
+__global__ void __launch_bounds__(THREADS, 2) k_esc(EscArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  EscSmem<T>& S = *reinterpret_cast<EscSmem<T>*>(smem_raw);
+  const int tid = threadIdx.x;
+  const int b = blockIdx.x;
+  const int32_t* __restrict__ arp = a.A.row_ptr;
+  const int32_t* __restrict__ acol = a.A.col;
+  const T* __restrict__ aval = reinterpret_cast<const T*>(a.A.val);
+  const int32_t* __restrict__ brp = a.B.row_ptr;
+  const int32_t* __restrict__ bcol = a.B.col;
+  const T* __restrict__ bval = reinterpret_cast<const T*>(a.B.val);
+  const int nzb = a.blk_nz_begin[b];
+  const int n_a = a.blk_nz_end[b] - nzb;
+  const int r0 = a.block_row_starts[b];
+  const int64_t rowsA = a.A.rows;
+
+  // ---------------- Fetch A (§3.2.1) ----------------
+  {
+    const int64_t r = (int64_t)r0 + tid;
+    S.rp_cache[tid] = r <= rowsA ? arp[r] : INT_MAX;
+    if (tid == 0) {
+      const int64_t r2 = (int64_t)r0 + THREADS;
+      S.rp_cache[THREADS] = r2 <= rowsA ? arp[r2] : INT_MAX;
+    }
+  }
+  __syncthreads();
+  int len[NNZ_PER_THREAD], row[NNZ_PER_THREAD];
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+    const int e = tid * NNZ_PER_THREAD + j;
+    if (e < n_a) {
+      const int nz = nzb + e;
+      const int k = acol[nz];
+      S.a_val[e] = aval[nz];
+      const int bs = brp[k];
+      S.a_bstart[e] = bs;
+      len[j] = brp[k + 1] - bs;
+      int r;
+      if (nz < S.rp_cache[THREADS]) {            // row within the cached window
+        int lo = 0, hi = THREADS - 1;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (S.rp_cache[mid] <= nz) lo = mid; else hi = mid - 1;
+        }
+        r = r0 + lo;
+      } else {                                    // many (empty) rows: search globally
+        int64_t lo = (int64_t)r0 + THREADS, hi = rowsA - 1;
+        while (lo < hi) {
+          const int64_t mid = (lo + hi + 1) >> 1;
+          if (arp[mid] <= nz) lo = mid; else hi = mid - 1;
+        }
+        r = (int)lo;
+      }
+      row[j] = r;
+    } else {
+      len[j] = 0;
+      row[j] = INT_MAX;
+    }
+    if (e < NPB) S.a_lrow[e] = row[j];
+  }
+  __syncthreads();
+  // dense local row ids: rank of the row among the block's rows
+  int f[NNZ_PER_THREAD], cnt = 0;
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+    const int e = tid * NNZ_PER_THREAD + j;
+    f[j] = (e < n_a) && (e == 0 || S.a_lrow[e - 1] != row[j]);
+    cnt += f[j];
+  }
+  int tot;
+  int run = block_exclusive_sum<int>(cnt, S.s.scratch, &tot);
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+    const int e = tid * NNZ_PER_THREAD + j;
+    run += f[j];
+    if (e < n_a) {
+      S.a_lrow[e] = run - 1;
+      if (f[j]) S.row_of[run - 1] = row[j];
+    }
+  }
+  wd_placework(len, S.wd, S.s.scratch);
+
+  EscState st{0, 0, 0, 0, 0, 0};
+  const int64_t pool_base = a.pool_off[b];
+  const int64_t desc_base = a.desc_off[b];
+  int size = S.wd[NPB];
+  while (size > 0) {
+    const int consume = min(CAP - st.kept, size);
+    int ares[ITEMS], bres[ITEMS];
+    wd_receivework(consume, S.wd, S.s.u.offsets, S.s.scratch, ares, bres);
+    const int size_after = S.wd[NPB];
+    // ---------------- expand (L340) ----------------
+    int col[ITEMS], lr[ITEMS];
+    T v[ITEMS];
+    int rmin = INT_MAX, rmax = INT_MIN, cmin = INT_MAX, cmax = INT_MIN;
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+      if (ares[i] >= 0) {
+        const int e = ares[i];
+        const int q = S.a_bstart[e] + bres[i];
+        col[i] = __ldg(bcol + q);
+        v[i] = S.a_val[e] * __ldg(bval + q);
+        lr[i] = S.a_lrow[e];
+        rmin = min(rmin, lr[i]); rmax = max(rmax, lr[i]);
+        cmin = min(cmin, col[i]); cmax = max(cmax, col[i]);
+      } else {
+        col[i] = 0; lr[i] = 0; v[i] = (T)0;
+      }
+    }
+    if (st.kept > 0) {
+      rmin = min(rmin, st.kept_lrow); rmax = max(rmax, st.kept_lrow);
+      cmin = min(cmin, st.kept_cmin); cmax = max(cmax, st.kept_cmax);
+    }
+    block_minmax4(rmin, rmax, cmin, cmax, S.s.scratch);
+    // dynamic bit reduction (L342-L344): only the row and column ranges present
+    const int rowbits = bit_width_u64((uint64_t)(rmax - rmin));
+    const int colbits = bit_width_u64((uint64_t)((int64_t)cmax - (int64_t)cmin));
+    if (rowbits + colbits + IDXBITS <= 32)
+      esc_iteration<uint32_t, T>(S, a, st, consume, size_after, ares, lr, col, v, rmin, cmin, rowbits, colbits,
+                                 pool_base, desc_base);
+    else
+      esc_iteration<uint64_t, T>(S, a, st, consume, size_after, ares, lr, col, v, rmin, cmin, rowbits, colbits,
+                                 pool_base, desc_base);
+    size = size_after;
+  }
+  if (tid == 0) a.nchunks[b] = st.seq;
+}
+
+template <typename T>
+static void launch_esc_t(const EscArgs& a, cudaStream_t st) {
+  const size_t smem = sizeof(EscSmem<T>);
+  cudaFuncSetAttribute(k_esc<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k_esc<T><<<a.nblocks, THREADS, smem, st>>>(a);
+}
+
+void launch_esc(const EscArgs& a, bool f64, cudaStream_t st) {
+  if (a.nblocks <= 0) return;
+  if (f64) launch_esc_t<double>(a, st); else launch_esc_t<float>(a, st);
+}
+
+}  // namespace acs
