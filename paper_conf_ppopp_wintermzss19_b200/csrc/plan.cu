@@ -262,6 +262,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->pool_val, (size_t)vbytes * products);
   ACS_ENSURE(p->descs, sizeof(ChunkDesc) * slots);
   ACS_ENSURE(p->row_count, sizeof(int32_t) * A->rows);
+  // scans later run over up to `slots` chunks / shared rows
+  ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * scan_tmp_elems(std::max<int64_t>(std::max(max_blocks, A->rows), slots) + 1));
   p->info.pool_bytes = (int64_t)(p->pool_col.bytes + p->pool_val.bytes);
   ACS_CUDA(cudaMemsetAsync(p->row_count.p, 0, sizeof(int32_t) * A->rows, st));
 
