@@ -271,7 +271,10 @@ __global__ void __launch_bounds__(THREADS, 2) k_esc(EscArgs a) {
                                  pool_base, desc_base);
     size = size_after;
   }
-  if (tid == 0) a.nchunks[b] = st.seq;
+  if (tid == 0) {
+    a.nchunks[b] = st.seq;
+    a.used[b] = (int32_t)st.wofs;
+  }
 }
 
 template <typename T>

@@ -46,6 +46,7 @@ struct EscArgs {
   void* pool_val;
   ChunkDesc* descs;
   int32_t* nchunks;             // per block
+  int32_t* used;                // per block: chunk elements written
   int32_t* row_count;           // per row of C
 };
 void launch_esc(const EscArgs& a, bool f64, cudaStream_t st);

@@ -67,7 +67,7 @@ struct acspgemm_plan_s {
   DevBuf seg, seg_rows, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base;
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, mscan, mtscan, group_of, gstart, merge_col, merge_val;
-  DevBuf cur_first, cur_last, err;
+  DevBuf cur_first, cur_last, err, bused, bused_scan;
   int64_t* h_scal = nullptr;     // pinned read-back buffer
   cudaEvent_t ev[NSTAGE_EV];
   bool ev_ok = false;
@@ -141,7 +141,7 @@ int64_t helper_bytes(acspgemm_plan p) {
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->descs, &p->dense, &p->sflag,
                   &p->spos, &p->shared, &p->row_count, &p->row_ptr, &p->scan_tmp, &p->kflag, &p->kpos,
                   &p->lmulti, &p->lpath, &p->lsearch, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
-                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err};
+                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan};
   int64_t t = 0;
   for (DevBuf* b : bs) t += (int64_t)b->bytes;
   return t;
@@ -227,6 +227,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->desc_off, sizeof(int64_t) * max_blocks);
   ACS_ENSURE(p->nchunks, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->chunk_base, sizeof(int64_t) * max_blocks);
+  ACS_ENSURE(p->bused, sizeof(int32_t) * max_blocks);
+  ACS_ENSURE(p->bused_scan, sizeof(int64_t) * max_blocks);
   const int64_t tmp_n = scan_tmp_elems(std::max<int64_t>(max_blocks, A->rows) * 2 + 1024);
   ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * tmp_n);
   int32_t* nblocks_dev = reinterpret_cast<int32_t*>(scal + 20);
@@ -282,6 +284,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.pool_val = p->pool_val.p;
   ea.descs = ptr<ChunkDesc>(p->descs);
   ea.nchunks = ptr<int32_t>(p->nchunks);
+  ea.used = ptr<int32_t>(p->bused);
   ea.row_count = ptr<int32_t>(p->row_count);
   launch_esc(ea, p->f64, st);
   tl_launches += nblocks > 0 ? 1 : 0;
@@ -294,7 +297,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->spos, sizeof(int64_t) * slots);
   ACS_ENSURE(p->shared, sizeof(SharedRow) * slots);
   launch_scan_i32(ptr<int32_t>(p->nchunks), ptr<int64_t>(p->chunk_base), nblocks, scal + 3, ptr<int64_t>(p->scan_tmp), st);
-  tl_launches += 3;
+  launch_scan_i32(ptr<int32_t>(p->bused), ptr<int64_t>(p->bused_scan), nblocks, scal + 5, ptr<int64_t>(p->scan_tmp), st);
+  tl_launches += 6;
   MergeState ms;
   ms.nblocks = (int32_t)nblocks;
   ms.desc_off = ptr<int64_t>(p->desc_off);
@@ -312,13 +316,13 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   launch_find_shared(ms, scal + 4, st);
   tl_launches += 1 + (slots > 0 ? 5 : 0);
   ACS_CUDA(cudaGetLastError());
-  if ((s = sync_read(p, scal + 3, 2, st)) != ACSPGEMM_OK) return s;
+  if ((s = sync_read(p, scal + 3, 3, st)) != ACSPGEMM_OK) return s;
   p->total_chunks = p->h_scal[0];
   p->nshared = p->h_scal[1];
   p->max_chunks = slots;
   p->info.nchunks = p->total_chunks;
   p->info.nshared = p->nshared;
-  p->info.chunk_elems = 0;
+  p->info.chunk_elems = p->h_scal[2];
   const int64_t nsh = p->nshared;
   int64_t nmulti = 0, npath = 0, nsearch = 0, merge_total = 0, ngroups = 0;
   if (nsh > 0) {
@@ -586,7 +590,7 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
                   &p->descs, &p->dense, &p->sflag, &p->spos, &p->shared, &p->row_count, &p->row_ptr,
                   &p->scan_tmp, &p->kflag, &p->kpos, &p->lmulti, &p->lpath, &p->lsearch, &p->mscan,
                   &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
-                  &p->cur_last, &p->err};
+                  &p->cur_last, &p->err, &p->bused, &p->bused_scan};
   for (DevBuf* b : bs) free_buf(*b);
   if (p->h_scal) cudaFreeHost(p->h_scal);
   if (p->ev_ok)
