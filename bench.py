@@ -43,7 +43,7 @@ CONFIGS = {
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="cuda", choices=["cuda", "reference"])
     ap.add_argument("--config", default="cfg2", choices=sorted(CONFIGS))
@@ -87,6 +87,9 @@ class ClockSampler:
                 self.lines.append(line.strip())
         self.thread = threading.Thread(target=reader, daemon=True)
         self.thread.start()
+        t0 = time.time()
+        while not self.lines and time.time() - t0 < 5.0:   # first sample before timing starts
+            time.sleep(0.02)
 
     def stop(self):
         if self.proc is None:
