@@ -11,19 +11,27 @@
 
 namespace acs {
 
-constexpr int THREADS = 256;                 // threads per CTA (L344)
-constexpr int ITEMS = 8;                     // sorted elements per thread (L556)
-constexpr int CAP = THREADS * ITEMS;         // products per local ESC iteration
+#ifndef ACS_THREADS
+#define ACS_THREADS 256
+#endif
+#ifndef ACS_ITEMS
+#define ACS_ITEMS 8
+#endif
+constexpr int THREADS = ACS_THREADS;         // threads per CTA (paper: 256, L344)
+constexpr int ITEMS = ACS_ITEMS;             // sorted elements per thread (paper: 8, L556)
+constexpr int CAP = THREADS * ITEMS;         // products per local ESC iteration (2048)
 constexpr int IDXBITS = 11;                  // log2(CAP): position bits in a sort word
-constexpr int NNZ_PER_THREAD = 2;            // A entries per thread (L344)
-constexpr int NPB = THREADS * NNZ_PER_THREAD;// NNZ_PER_BLOCK (Alg. 1, Alg. 2)
-constexpr int KEEP = 4 * THREADS;            // max kept elements of the last row (L556)
+constexpr int NPB = 512;                     // NNZ_PER_BLOCK (Alg. 1, Alg. 2; L556 "256/512")
+constexpr int NNZ_PER_THREAD = NPB / THREADS;// A entries per thread
+constexpr int KEEP_PER_THREAD = 4;           // "keeps up to 4 elements per thread" (L556)
+constexpr int KEEP = KEEP_PER_THREAD * THREADS; // max kept elements of the last row
 constexpr int RADIX_BITS = 5;                // digit width of one radix-sort pass
 constexpr int DEFAULT_SEGMENTS = 8;          // canonical segments
 constexpr int MAX_SEGMENTS = 64;
 constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)
 static_assert((1 << IDXBITS) == CAP, "IDXBITS must be log2(CAP)");
 static_assert(KEEP <= CAP / 2, "kept row must leave room for new products");
+static_assert(NPB % THREADS == 0, "NPB must be a multiple of THREADS");
 
 // A chunk of C (§3.2.4: "each chunk holds its starting row, element
 // count and number of elements in the first and last row"; the chunk id (block,

@@ -27,23 +27,22 @@ struct EscSmem {
   int a_lrow[NPB];
   int row_of[NPB];
   int wd[NPB + 1];
-  int rp_cache[THREADS + 1];
-  int kept_col[KEEP];
-  T kept_val[KEEP];
+  int rp_cache[NPB + 1];
 };
 
 struct EscState {
-  int kept, kept_lrow, kept_cmin, kept_cmax;
+  int kept, kofs, kept_lrow, kept_cmin, kept_cmax;  // kept row lives in the staging area
   int seq;
   int64_t wofs;
 };
 
-// One local ESC iteration after expansion: build words, sort, compact, emit.
+// One local ESC iteration after expansion (values already at s.vals[pos]): build the
+// sort words, sort, compact (Alg. 3), emit completed rows as a chunk, keep the last row.
 template <typename Word, typename T>
 __device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, EscState& st, int consume,
-                                              int size_after, const int (&ares)[ITEMS], const int (&lr)[ITEMS],
-                                              const int (&col)[ITEMS], const T (&v)[ITEMS], int rmin, int cmin,
-                                              int rowbits, int colbits, int64_t pool_base, int64_t desc_base) {
+                                              int size_after, const int (&ares)[ITEMS], const int (&col)[ITEMS],
+                                              const int (&kc)[KEEP_PER_THREAD], int rmin, int cmin, int rowbits,
+                                              int colbits, int64_t pool_base, int64_t desc_base) {
   const int tid = threadIdx.x;
   const int kept = st.kept;
   const int n = kept + consume;
@@ -53,36 +52,28 @@ __device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, E
   for (int i = 0; i < ITEMS; ++i) {
     if (ares[i] >= 0) {
       const int pos = kept + i * THREADS + tid;
-      const Word key = ((Word)(lr[i] - rmin) << colbits) | (Word)(col[i] - cmin);
-      sw[pos] = (key << IDXBITS) | (Word)pos;
-      S.s.vals[pos] = v[i];
+      const Word key = ((Word)(S.a_lrow[ares[i]] - rmin) << colbits) | (Word)(col[i] - cmin);
+      sw[pad32(pos)] = (key << IDXBITS) | (Word)pos;
     }
   }
-  for (int p = tid; p < kept; p += THREADS) {
-    const Word key = ((Word)(st.kept_lrow - rmin) << colbits) | (Word)(S.kept_col[p] - cmin);
-    sw[p] = (key << IDXBITS) | (Word)p;
-    S.s.vals[p] = S.kept_val[p];
-  }
-  for (int p = n + tid; p < CAP; p += THREADS) sw[p] = ~(Word)0;
-  __syncthreads();
-
-  CElem<Word, T> x[ITEMS];
-  sort_and_scan<Word, T>(S.s, n, rowbits + colbits, colbits, x);
-
-  int* misc = S.s.misc;
-  if (tid == (n - 1) / ITEMS) {
-    const int i = (n - 1) % ITEMS;
 #pragma unroll
-    for (int q = 0; q < ITEMS; ++q) {
-      if (q == i) {
-        misc[0] = st_count(x[q].state);
-        misc[1] = st_row_count(x[q].state);
-        misc[2] = (int)(x[q].key >> colbits);
-      }
+  for (int j = 0; j < KEEP_PER_THREAD; ++j) {
+    const int p = j * THREADS + tid;
+    if (p < kept) {
+      const Word key = ((Word)(st.kept_lrow - rmin) << colbits) | (Word)(kc[j] - cmin);
+      sw[pad32(p)] = (key << IDXBITS) | (Word)p;
     }
   }
+  for (int p = n + tid; p < CAP; p += THREADS) sw[pad32(p)] = ~(Word)0;
   __syncthreads();
-  const int total = misc[0], rc_last = misc[1], lastrel = misc[2];
+
+  Word k[ITEMS];
+  T ev[ITEMS];
+  load_and_sort<Word, T>(S.s, rowbits + colbits, k);
+  const ScanCtx<Word, T> ctx = compaction_prepare<Word, T>(S.s, k, n, colbits, ev);
+  const int total = st_count(ctx.total.state);
+  const int rc_last = st_row_count(ctx.total.state);
+  const int lastrel = (int)(ctx.total.key >> colbits);
   // keep the last row for the next iteration (L366) unless the block is done or the
   // row no longer fits the kept budget (reading R13: then it is written as a partial
   // chunk and merged later)
@@ -90,29 +81,24 @@ __device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, E
   const int nchunk = total - (keep ? rc_last : 0);
   int* stage_col = reinterpret_cast<int*>(S.s.words);
   T* stage_val = S.s.vals;
+  int* misc = S.s.misc;
   const Word colmask = colbits ? (((Word)1 << colbits) - (Word)1) : (Word)0;
-#pragma unroll
-  for (int i = 0; i < ITEMS; ++i) {
-    const uint32_t s = x[i].state;
-    if (s & 1u) {
-      const int p = st_count(s) - 1;
-      const int c = cmin + (int)(x[i].key & colmask);
-      const int rel = (int)(x[i].key >> colbits);
-      if (p < nchunk) {
-        stage_col[p] = c;
-        stage_val[p] = x[i].val;
-        if (st_row_end(s)) {
-          const int rc = st_row_count(s);
-          a.row_count[S.row_of[rmin + rel]] = rc;        // per-row counter (L362)
-          if (rel == 0) misc[3] = rc;
-          if (p == nchunk - 1) { misc[4] = rel; misc[5] = rc; }
-        }
-      } else {
-        S.kept_col[p - nchunk] = c;
-        S.kept_val[p - nchunk] = x[i].val;
-      }
+  // compacted element p goes to staging slot p: [0, nchunk) is the chunk, the kept
+  // row stays at [nchunk, total) for the next iteration
+  compaction_emit<Word, T>(k, ev, n, colbits, ctx, [&](int, Word key, T val, uint32_t state, bool run_end,
+                                                       bool row_end) {
+    if (!run_end) return;
+    const int p = st_count(state) - 1;
+    stage_col[p] = cmin + (int)(key & colmask);
+    stage_val[p] = val;
+    if (row_end && p < nchunk) {
+      const int rc = st_row_count(state);
+      const int rel = (int)(key >> colbits);
+      a.row_count[S.row_of[rmin + rel]] = rc;        // per-row counter (L362)
+      if (rel == 0) misc[3] = rc;
+      if (p == nchunk - 1) { misc[4] = rel; misc[5] = rc; }
     }
-  }
+  });
   __syncthreads();
   if (nchunk > 0) {
     // chunk write through shared memory for coalescing (L424-L426)
@@ -137,16 +123,17 @@ __device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, E
     st.wofs += nchunk;
   }
   st.kept = keep ? rc_last : 0;
+  st.kofs = nchunk;
   if (keep) {
     st.kept_lrow = rmin + lastrel;
-    st.kept_cmin = S.kept_col[0];
-    st.kept_cmax = S.kept_col[st.kept - 1];
+    st.kept_cmin = stage_col[nchunk];
+    st.kept_cmax = stage_col[total - 1];
   }
   __syncthreads();
 }
 
 template <typename T>
-__global__ void __launch_bounds__(THREADS, 2) k_esc(EscArgs a) {
+__global__ void __launch_bounds__(THREADS, 3) k_esc(EscArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   EscSmem<T>& S = *reinterpret_cast<EscSmem<T>*>(smem_raw);
   const int tid = threadIdx.x;
@@ -163,13 +150,10 @@ __global__ void __launch_bounds__(THREADS, 2) k_esc(EscArgs a) {
   const int64_t rowsA = a.A.rows;
 
   // ---------------- Fetch A (§3.2.1) ----------------
-  {
-    const int64_t r = (int64_t)r0 + tid;
-    S.rp_cache[tid] = r <= rowsA ? arp[r] : INT_MAX;
-    if (tid == 0) {
-      const int64_t r2 = (int64_t)r0 + THREADS;
-      S.rp_cache[THREADS] = r2 <= rowsA ? arp[r2] : INT_MAX;
-    }
+  // row_ptr[r0 .. r0+NPB] covers every row of the block unless it has empty rows
+  for (int t = tid; t <= NPB; t += THREADS) {
+    const int64_t r = (int64_t)r0 + t;
+    S.rp_cache[t] = r <= rowsA ? arp[r] : INT_MAX;
   }
   __syncthreads();
   int len[NNZ_PER_THREAD], row[NNZ_PER_THREAD];
@@ -184,15 +168,15 @@ __global__ void __launch_bounds__(THREADS, 2) k_esc(EscArgs a) {
       S.a_bstart[e] = bs;
       len[j] = brp[k + 1] - bs;
       int r;
-      if (nz < S.rp_cache[THREADS]) {            // row within the cached window
-        int lo = 0, hi = THREADS - 1;
+      if (nz < S.rp_cache[NPB]) {                 // row within the cached window
+        int lo = 0, hi = NPB - 1;
         while (lo < hi) {
           const int mid = (lo + hi + 1) >> 1;
           if (S.rp_cache[mid] <= nz) lo = mid; else hi = mid - 1;
         }
         r = r0 + lo;
       } else {                                    // many (empty) rows: search globally
-        int64_t lo = (int64_t)r0 + THREADS, hi = rowsA - 1;
+        int64_t lo = (int64_t)r0 + NPB, hi = rowsA - 1;
         while (lo < hi) {
           const int64_t mid = (lo + hi + 1) >> 1;
           if (arp[mid] <= nz) lo = mid; else hi = mid - 1;
@@ -228,18 +212,32 @@ __global__ void __launch_bounds__(THREADS, 2) k_esc(EscArgs a) {
   }
   wd_placework(len, S.wd, S.s.scratch);
 
-  EscState st{0, 0, 0, 0, 0, 0};
+  EscState st{0, 0, 0, 0, 0, 0, 0};
   const int64_t pool_base = a.pool_off[b];
   const int64_t desc_base = a.desc_off[b];
   int size = S.wd[NPB];
   while (size > 0) {
     const int consume = min(CAP - st.kept, size);
+    // the kept row sits in the staging area, which the new values overwrite: pull it
+    // into registers first (receivework's barriers order this before the writes)
+    int kc[KEEP_PER_THREAD];
+    T kv[KEEP_PER_THREAD];
+#pragma unroll
+    for (int j = 0; j < KEEP_PER_THREAD; ++j) {
+      const int p = j * THREADS + tid;
+      if (p < st.kept) {
+        kc[j] = reinterpret_cast<int*>(S.s.words)[st.kofs + p];
+        kv[j] = S.s.vals[st.kofs + p];
+      } else {
+        kc[j] = 0;
+        kv[j] = (T)0;
+      }
+    }
     int ares[ITEMS], bres[ITEMS];
     wd_receivework(consume, S.wd, S.s.u.offsets, S.s.scratch, ares, bres);
     const int size_after = S.wd[NPB];
     // ---------------- expand (L340) ----------------
-    int col[ITEMS], lr[ITEMS];
-    T v[ITEMS];
+    int col[ITEMS];
     int rmin = INT_MAX, rmax = INT_MIN, cmin = INT_MAX, cmax = INT_MIN;
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
@@ -247,13 +245,18 @@ __global__ void __launch_bounds__(THREADS, 2) k_esc(EscArgs a) {
         const int e = ares[i];
         const int q = S.a_bstart[e] + bres[i];
         col[i] = __ldg(bcol + q);
-        v[i] = S.a_val[e] * __ldg(bval + q);
-        lr[i] = S.a_lrow[e];
-        rmin = min(rmin, lr[i]); rmax = max(rmax, lr[i]);
+        S.s.vals[st.kept + i * THREADS + tid] = S.a_val[e] * __ldg(bval + q);
+        const int lr = S.a_lrow[e];
+        rmin = min(rmin, lr); rmax = max(rmax, lr);
         cmin = min(cmin, col[i]); cmax = max(cmax, col[i]);
       } else {
-        col[i] = 0; lr[i] = 0; v[i] = (T)0;
+        col[i] = 0;
       }
+    }
+#pragma unroll
+    for (int j = 0; j < KEEP_PER_THREAD; ++j) {
+      const int p = j * THREADS + tid;
+      if (p < st.kept) S.s.vals[p] = kv[j];
     }
     if (st.kept > 0) {
       rmin = min(rmin, st.kept_lrow); rmax = max(rmax, st.kept_lrow);
@@ -264,10 +267,10 @@ __global__ void __launch_bounds__(THREADS, 2) k_esc(EscArgs a) {
     const int rowbits = bit_width_u64((uint64_t)(rmax - rmin));
     const int colbits = bit_width_u64((uint64_t)((int64_t)cmax - (int64_t)cmin));
     if (rowbits + colbits + IDXBITS <= 32)
-      esc_iteration<uint32_t, T>(S, a, st, consume, size_after, ares, lr, col, v, rmin, cmin, rowbits, colbits,
+      esc_iteration<uint32_t, T>(S, a, st, consume, size_after, ares, col, kc, rmin, cmin, rowbits, colbits,
                                  pool_base, desc_base);
     else
-      esc_iteration<uint64_t, T>(S, a, st, consume, size_after, ares, lr, col, v, rmin, cmin, rowbits, colbits,
+      esc_iteration<uint64_t, T>(S, a, st, consume, size_after, ares, col, kc, rmin, cmin, rowbits, colbits,
                                  pool_base, desc_base);
     size = size_after;
   }

@@ -4,10 +4,15 @@
 //   * a stable block radix sort over packed (key | position) words with dynamic bit
 //     range (§3.2.3),
 //   * the compaction scan with the CombineScanOperator (Alg. 3).
+// Shared-memory arrays that are read in blocked order (thread t reads t*ITEMS + i) use
+// one padding word per 32 (`pad32`) so those reads are bank-conflict free.
 #pragma once
 #include "common.cuh"
 
 namespace acs {
+
+__device__ __forceinline__ int pad32(int i) { return i + (i >> 5); }
+constexpr int CAP_PAD = CAP + CAP / 32;
 
 // =====================================================================
 // Alg. 2 — local work distribution.  WDState[NPB+1] lives in shared memory.
@@ -34,19 +39,23 @@ __device__ __forceinline__ void wd_placework(const int (&len)[NNZ_PER_THREAD], i
 // receivework (lines 10-38) for `consume` (<= size()) products.  On return thread t
 // holds products c = i*THREADS + t (striped, line 25) as (ares[i], bres[i]); ares = -1
 // marks c >= consume.  Bres is the offset inside the A entry's B row counted down from
-// the row's remaining end (line 29).  `offsets` needs CAP ints.
+// the row's remaining end (line 29).  `offsets` needs CAP_PAD ints.
 __device__ __forceinline__ void wd_receivework(int consume, int* wd, int* offsets, int* scratch,
                                                int (&ares)[ITEMS], int (&bres)[ITEMS]) {
   const int tid = threadIdx.x;
   // line 14: clear(Offsets) — 0 is the identity of the max scan (reading R5)
-  for (int c = tid; c < consume; c += THREADS) offsets[c] = 0;
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    const int c = i * THREADS + tid;
+    if (c < consume) offsets[pad32(c)] = 0;
+  }
   __syncthreads();
   // lines 16-20: mark the first product of every entry that starts inside the draw
 #pragma unroll
   for (int i = 0; i < NNZ_PER_THREAD; ++i) {
     const int e = i * THREADS + tid;
     const int a = wd[e], an = wd[e + 1];
-    if (a < consume && a != an) offsets[a] = e;
+    if (a < consume && a != an) offsets[pad32(a)] = e;
   }
   __syncthreads();
   // line 24: block max scan, blocked layout
@@ -55,14 +64,14 @@ __device__ __forceinline__ void wd_receivework(int consume, int* wd, int* offset
 #pragma unroll
   for (int i = 0; i < ITEMS; ++i) {
     const int c = tid * ITEMS + i;
-    m = max(m, c < consume ? offsets[c] : 0);
+    m = max(m, c < consume ? offsets[pad32(c)] : 0);
     loc[i] = m;
   }
   const int ex = block_exclusive_max(m, scratch);
 #pragma unroll
   for (int i = 0; i < ITEMS; ++i) {
     const int c = tid * ITEMS + i;
-    if (c < consume) offsets[c] = max(ex, loc[i]);
+    if (c < consume) offsets[pad32(c)] = max(ex, loc[i]);
   }
   __syncthreads();
   // line 25: blocked -> striped; lines 26-32
@@ -70,7 +79,7 @@ __device__ __forceinline__ void wd_receivework(int consume, int* wd, int* offset
   for (int i = 0; i < ITEMS; ++i) {
     const int c = i * THREADS + tid;
     if (c < consume) {
-      const int e = offsets[c];
+      const int e = offsets[pad32(c)];
       ares[i] = e;
       bres[i] = wd[e + 1] - c - 1;
     } else {
@@ -93,37 +102,41 @@ __device__ __forceinline__ void wd_receivework(int consume, int* wd, int* offset
 // A word is  key << IDXBITS | position.  Sorting only the key bits with a stable LSD
 // radix sort keeps equal keys in position order, i.e. the expansion order (kept
 // elements first, then products by A entry) that the paper's stable sort preserves
-// for bit-stable sums (L198).  Ranking uses per-thread 16-bit digit counters packed
-// two per word (RADIX_BITS = 5 -> 32 digits = 16 counter lanes x 2 halves), a raking
-// exclusive scan over (lane, thread) order, and a scatter through shared memory.
+// for bit-stable sums (L198).  Ranking: per-thread 16-bit digit counters packed two per
+// word (RADIX_BITS = 5 -> 32 digits = 16 counter lanes x 2 halves), a raking exclusive
+// scan over (lane, thread) order, a scatter through shared memory.  Five barriers per
+// pass.  Words live at pad32(index).
 // =====================================================================
 
 constexpr int CNT_LANES = 16;
-constexpr int CNT_WORDS = CNT_LANES * THREADS;
-constexpr int CNT_PADDED = CNT_WORDS + CNT_WORDS / 32;
-constexpr int RAKE = CNT_WORDS / THREADS;
+constexpr int LANE_STRIDE = THREADS + THREADS / 32;         // padded words per counter lane
+constexpr int CNT_PADDED = CNT_LANES * LANE_STRIDE;
+constexpr int RAKE = CNT_LANES;                             // words per thread in the raking scan
 static_assert(RADIX_BITS <= 5, "two 16-bit halves x 16 lanes");
-
-__device__ __forceinline__ int cpad(int w) { return w + (w >> 5); }
+static_assert(THREADS % 32 == 0 && RAKE <= 32 && 32 % RAKE == 0, "raking layout");
+static_assert(ITEMS <= 32 && 32 % ITEMS == 0, "blocked items must not straddle padding");
 
 template <typename Word>
 __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words, uint32_t* s_cnt,
-                                                 uint32_t* s_scan, int begin_bit, int end_bit) {
-  const int tid = threadIdx.x;
+                                                 uint32_t* s_warp, int begin_bit, int end_bit) {
+  const int tid = threadIdx.x, lane = lane_id(), w = warp_id();
   uint16_t* c16 = reinterpret_cast<uint16_t*>(s_cnt);
+  const int tb2 = 2 * (tid + (tid >> 5));                   // my column in every counter lane
+  const int seg0 = pad32(tid * RAKE);                       // my raking segment (contiguous)
+  const int bb = pad32(tid * ITEMS);                        // my blocked items (contiguous)
+  if (begin_bit >= end_bit) return;
+#pragma unroll
+  for (int j = 0; j < RAKE; ++j) s_cnt[seg0 + j] = 0u;
+  __syncthreads();
   for (int bit = begin_bit; bit < end_bit; bit += RADIX_BITS) {
     const int nb = min(RADIX_BITS, end_bit - bit);
     const uint32_t mask = (1u << nb) - 1u;
-#pragma unroll
-    for (int j = 0; j < RAKE; ++j) s_cnt[cpad(tid * RAKE + j)] = 0u;
-    __syncthreads();
     int cidx[ITEMS];
     uint32_t pre[ITEMS];
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const uint32_t d = (uint32_t)(k[i] >> bit) & mask;
-      const int W = (int)(d & 15u) * THREADS + tid;
-      cidx[i] = cpad(W) * 2 + (int)(d >> 4);
+      cidx[i] = (int)(d & 15u) * (2 * LANE_STRIDE) + (int)(d >> 4) + tb2;
       pre[i] = c16[cidx[i]];
       c16[cidx[i]] = (uint16_t)(pre[i] + 1u);
     }
@@ -131,21 +144,40 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
     uint32_t seg[RAKE];
     uint32_t sum = 0;
 #pragma unroll
-    for (int j = 0; j < RAKE; ++j) { seg[j] = s_cnt[cpad(tid * RAKE + j)]; sum += seg[j]; }
-    uint32_t total;
-    const uint32_t excl = block_exclusive_sum<uint32_t>(sum, s_scan, &total);
-    uint32_t run = excl + ((total & 0xFFFFu) << 16);   // digits 16..31 follow all of 0..15
+    for (int j = 0; j < RAKE; ++j) { seg[j] = s_cnt[seg0 + j]; sum += seg[j]; }
+    uint32_t inc = sum;
 #pragma unroll
-    for (int j = 0; j < RAKE; ++j) { const uint32_t v = seg[j]; s_cnt[cpad(tid * RAKE + j)] = run; run += v; }
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, d);
+      if (lane >= d) inc += y;
+    }
+    if (lane == 31) s_warp[w] = inc;
     __syncthreads();
-    int rank[ITEMS];
+    uint32_t wpre = 0, grand = 0;
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) rank[i] = (int)c16[cidx[i]] + (int)pre[i];
+    for (int q = 0; q < THREADS / 32; ++q) {
+      const uint32_t t = s_warp[q];
+      wpre += q < w ? t : 0u;
+      grand += t;
+    }
+    // digits 16..31 (high halves) follow all of 0..15 (low halves)
+    uint32_t run = wpre + inc - sum + ((grand & 0xFFFFu) << 16);
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) s_words[rank[i]] = k[i];
+    for (int j = 0; j < RAKE; ++j) { const uint32_t v = seg[j]; s_cnt[seg0 + j] = run; run += v; }
     __syncthreads();
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) k[i] = s_words[tid * ITEMS + i];
+    for (int i = 0; i < ITEMS; ++i) {
+      const int rank = (int)c16[cidx[i]] + (int)pre[i];
+      s_words[pad32(rank)] = k[i];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) k[i] = s_words[bb + i];
+    if (bit + RADIX_BITS < end_bit) {
+#pragma unroll
+      for (int j = 0; j < RAKE; ++j) s_cnt[seg0 + j] = 0u;
+      __syncthreads();
+    }
   }
 }
 
@@ -189,42 +221,6 @@ __device__ __forceinline__ CElem<Key, T> shfl_up_elem(const CElem<Key, T>& x, in
   return y;
 }
 
-// Inclusive block scan of ITEMS elements per thread (blocked layout) with the fixed
-// tree: thread-sequential, warp Kogge-Stone, then the warps in order.  The tree is
-// fixed by (THREADS, ITEMS), so results are bit-stable run to run.
-template <typename Key, typename T>
-__device__ __forceinline__ void block_compaction_scan(CElem<Key, T> (&x)[ITEMS], int colbits,
-                                                      CElem<Key, T>* s_warp) {
-  const int lane = lane_id(), w = warp_id();
-#pragma unroll
-  for (int i = 1; i < ITEMS; ++i) x[i] = combine_op(x[i - 1], x[i], colbits);
-  CElem<Key, T> inc = x[ITEMS - 1];
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    CElem<Key, T> y = shfl_up_elem(inc, d);
-    if (lane >= d) inc = combine_op(y, inc, colbits);
-  }
-  CElem<Key, T> ex = shfl_up_elem(inc, 1);
-  if (lane == 31) s_warp[w] = inc;
-  __syncthreads();
-  bool has = false;
-  CElem<Key, T> pre;
-  if (w > 0) {
-    pre = s_warp[0];
-    for (int j = 1; j < w; ++j) pre = combine_op(pre, s_warp[j], colbits);
-    has = true;
-  }
-  if (lane > 0) {
-    pre = has ? combine_op(pre, ex, colbits) : ex;
-    has = true;
-  }
-  if (has) {
-#pragma unroll
-    for (int i = 0; i < ITEMS; ++i) x[i] = combine_op(pre, x[i], colbits);
-  }
-  __syncthreads();
-}
-
 __device__ __forceinline__ int st_count(uint32_t s) { return (int)((s >> 1) & 0x7FFFu); }
 __device__ __forceinline__ int st_row_count(uint32_t s) { return (int)((s >> 17) & 0x7FFFu); }
 __device__ __forceinline__ bool st_run_end(uint32_t s) { return s & 1u; }
@@ -234,54 +230,167 @@ __device__ __forceinline__ bool st_row_end(uint32_t s) { return (s >> 16) & 1u; 
 template <typename T>
 struct SortSmem {
   union {
-    int offsets[CAP];                 // Alg. 2 Offsets
+    int offsets[CAP_PAD];             // Alg. 2 Offsets (padded)
     uint32_t cnt[CNT_PADDED];         // radix counters
-    int wprefix[CAP + 1];             // merge window prefix
+    int wprefix[CAP + 1];             // merge window prefix / path samples
   } u;
-  uint64_t words[CAP];                // sort buffer (uint32 words use the first half);
-                                      // reused as int32 staging of output columns
-  T vals[CAP];                        // values by position; reused as output staging
+  uint64_t words[CAP_PAD];            // sort buffer at pad32(i) (uint32 words use the first
+                                      // half); after the sort: int32 staging of output
+                                      // columns at plain index p
+  T vals[CAP];                        // values by position; after the sort: output staging
   CElem<uint64_t, T> warp_agg[THREADS / 32];
-  uint32_t scan32[THREADS / 32 + 1];
+  uint8_t warp_has[THREADS / 32];
+  uint32_t swarp[THREADS / 32];
   int scratch[40];
   int misc[16];
 };
 
-// Load the sorted words (blocked), run the compaction scan and leave per element
-// (key, run sum, state).  Words in s.words[0..CAP) hold key<<IDXBITS|pos, positions
-// >= n are padding (all ones) and sort last.
+// The compaction scan (Alg. 3) over the sorted words of a thread (blocked layout).
+// Within a thread the scan is a left fold; because the input is sorted, applying the
+// CombineScanOperator to a running element and the next item only needs the previous
+// item's run-end / row-end flags (a.key == b.key  <=>  previous item is not a run end;
+// equalRow  <=>  previous item is not a row end).  Across threads the operator itself
+// combines the per-thread aggregates (warp Kogge-Stone, then the warps in order).
+//   prepare: flags, values (into registers), the thread aggregate, the block scan of the
+//            aggregates; returns the carry-in and the block total (element n-1).
+//   emit:    re-folds the thread's items from the carry and calls
+//            f(idx, key, value, state, run_end, row_end) for every valid element.
+// The tree is fixed by (THREADS, ITEMS): results are bit-stable run to run.
 template <typename Word, typename T>
-__device__ __forceinline__ void sort_and_scan(SortSmem<T>& s, int n, int keybits, int colbits,
-                                              CElem<Word, T> (&x)[ITEMS]) {
-  Word* sw = reinterpret_cast<Word*>(s.words);
-  Word k[ITEMS];
-#pragma unroll
-  for (int i = 0; i < ITEMS; ++i) k[i] = sw[threadIdx.x * ITEMS + i];
-  block_radix_sort<Word>(k, sw, s.u.cnt, s.scan32, IDXBITS, IDXBITS + keybits);
-  // after the last pass the sorted words are also in sw (blocked order); with zero
-  // passes sw already is the input order
+struct ScanCtx {
+  CElem<Word, T> carry;
+  bool has_carry;
+  CElem<Word, T> total;
+  uint32_t flags;        // bit 2i: run end of item i, bit 2i+1: row end
+};
+
+__device__ __forceinline__ uint32_t init_state(bool run_end, bool row_end) {
+  return row_end ? ST_END_ROW : (run_end ? ST_END_COMP : 0u);
+}
+
+template <typename Word, typename T>
+__device__ __forceinline__ ScanCtx<Word, T> compaction_prepare(SortSmem<T>& s, const Word (&k)[ITEMS], int n,
+                                                                int colbits, T (&ev)[ITEMS]) {
+  const int lane = lane_id(), w = warp_id();
+  const Word* sw = reinterpret_cast<const Word*>(s.words);
   const Word posmask = (Word)(CAP - 1);
+  const int base = threadIdx.x * ITEMS;
+  ScanCtx<Word, T> ctx;
+  uint32_t flags = 0;
+  T val = (T)0;
+  uint32_t state = 0;
 #pragma unroll
   for (int i = 0; i < ITEMS; ++i) {
-    const int idx = threadIdx.x * ITEMS + i;
+    const int idx = base + i;
     const Word key = k[i] >> IDXBITS;
     Word nkey;
     if (i + 1 < ITEMS) nkey = k[i + 1] >> IDXBITS;
-    else nkey = (idx + 1 < CAP) ? (sw[idx + 1] >> IDXBITS) : key;
-    const bool valid = idx < n;
-    const bool last = idx == n - 1;
-    x[i].key = valid ? key : ~(Word)0;
-    x[i].val = valid ? s.vals[(int)(k[i] & posmask)] : (T)0;
-    uint32_t st = 0;
-    if (valid) {
-      const bool run_end = last || nkey != key;
-      const bool row_end = last || (nkey >> colbits) != (key >> colbits);
-      st = row_end ? ST_END_ROW : (run_end ? ST_END_COMP : 0u);
+    else nkey = (idx + 1 < CAP) ? (sw[pad32(idx + 1)] >> IDXBITS) : key;
+    const bool last = idx >= n - 1;
+    const bool run_end = last || nkey != key;
+    const bool row_end = last || (nkey >> colbits) != (key >> colbits);
+    flags |= ((uint32_t)run_end << (2 * i)) | ((uint32_t)row_end << (2 * i + 1));
+    ev[i] = idx < n ? s.vals[(int)(k[i] & posmask)] : (T)0;
+    if (i == 0) {
+      val = ev[0];
+      state = init_state(run_end, row_end);
+    } else if (idx < n) {
+      const bool prun = (flags >> (2 * i - 2)) & 1u, prow = (flags >> (2 * i - 1)) & 1u;
+      val = prun ? ev[i] : val + ev[i];
+      state = (prow ? (state & 0x0000FFFEu) : (state & 0xFFFEFFFEu)) + init_state(run_end, row_end);
     }
-    x[i].state = st;
   }
-  __syncthreads();   // all reads of words / vals done
-  block_compaction_scan<Word, T>(x, colbits, reinterpret_cast<CElem<Word, T>*>(s.warp_agg));
+  ctx.flags = flags;
+  const bool has = base < n;
+  CElem<Word, T> agg;
+  agg.key = k[min(ITEMS - 1, max(0, n - 1 - base))] >> IDXBITS;
+  agg.val = val;
+  agg.state = state;
+  // warp inclusive scan of (has, agg)
+  CElem<Word, T> inc = agg;
+  bool hinc = has;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    CElem<Word, T> y = shfl_up_elem(inc, d);
+    const bool hy = __shfl_up_sync(0xffffffffu, (int)hinc, d) != 0;
+    if (lane >= d && hy) {
+      inc = hinc ? combine_op(y, inc, colbits) : y;
+      hinc = true;
+    }
+  }
+  CElem<Word, T> ex = shfl_up_elem(inc, 1);
+  const bool hex = __shfl_up_sync(0xffffffffu, (int)hinc, 1) != 0 && lane > 0;
+  CElem<Word, T>* wagg = reinterpret_cast<CElem<Word, T>*>(s.warp_agg);
+  if (lane == 31) {
+    wagg[w] = inc;
+    s.warp_has[w] = hinc;
+  }
+  __syncthreads();
+  CElem<Word, T> wp, tot;
+  bool hwp = false, htot = false;
+#pragma unroll
+  for (int q = 0; q < THREADS / 32; ++q) {
+    if (s.warp_has[q]) {
+      const CElem<Word, T> v = wagg[q];
+      if (q < w) { wp = hwp ? combine_op(wp, v, colbits) : v; hwp = true; }
+      tot = htot ? combine_op(tot, v, colbits) : v;
+      htot = true;
+    }
+  }
+  if (hwp && hex) { ctx.carry = combine_op(wp, ex, colbits); ctx.has_carry = true; }
+  else if (hwp) { ctx.carry = wp; ctx.has_carry = true; }
+  else if (hex) { ctx.carry = ex; ctx.has_carry = true; }
+  else { ctx.has_carry = false; }
+  ctx.total = tot;
+  __syncthreads();
+  return ctx;
+}
+
+// (prepare ends with a barrier: after it the sort buffers may be overwritten)
+template <typename Word, typename T, typename F>
+__device__ __forceinline__ void compaction_emit(const Word (&k)[ITEMS], const T (&ev)[ITEMS], int n, int colbits,
+                                                const ScanCtx<Word, T>& ctx, F&& f) {
+  const int base = threadIdx.x * ITEMS;
+  T val = (T)0;
+  uint32_t state = 0;
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    const int idx = base + i;
+    if (idx < n) {
+      const Word key = k[i] >> IDXBITS;
+      const bool run_end = (ctx.flags >> (2 * i)) & 1u;
+      const bool row_end = (ctx.flags >> (2 * i + 1)) & 1u;
+      const uint32_t st0 = init_state(run_end, row_end);
+      if (i == 0) {
+        if (ctx.has_carry) {
+          const bool eq_key = ctx.carry.key == key;
+          const bool eq_row = (ctx.carry.key >> colbits) == (key >> colbits);
+          val = eq_key ? ctx.carry.val + ev[0] : ev[0];
+          state = (eq_row ? (ctx.carry.state & 0xFFFEFFFEu) : (ctx.carry.state & 0x0000FFFEu)) + st0;
+        } else {
+          val = ev[0];
+          state = st0;
+        }
+      } else {
+        const bool prun = (ctx.flags >> (2 * i - 2)) & 1u, prow = (ctx.flags >> (2 * i - 1)) & 1u;
+        val = prun ? ev[i] : val + ev[i];
+        state = (prow ? (state & 0x0000FFFEu) : (state & 0xFFFEFFFEu)) + st0;
+      }
+      f(idx, key, val, state, run_end, row_end);
+    }
+  }
+}
+
+// Load the n input words (written at pad32(pos), padding = all ones beyond n), sort the
+// key bits.  On return k holds the sorted words of this thread (blocked) and s.words the
+// whole sorted array at pad32(index).
+template <typename Word, typename T>
+__device__ __forceinline__ void load_and_sort(SortSmem<T>& s, int keybits, Word (&k)[ITEMS]) {
+  Word* sw = reinterpret_cast<Word*>(s.words);
+  const int bb = pad32(threadIdx.x * ITEMS);      // ITEMS divides 32: no padding inside
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) k[i] = sw[bb + i];
+  block_radix_sort<Word>(k, sw, s.u.cnt, s.swarp, IDXBITS, IDXBITS + keybits);
 }
 
 }  // namespace acs

@@ -474,7 +474,7 @@ acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t 
 __global__ void k_debug_wd(const int32_t* lengths, int nentries, const int32_t* draws, int ndraws, int32_t* ares_out,
                            int32_t* bres_out, int32_t* rem_out) {
   __shared__ int wd[NPB + 1];
-  __shared__ int offsets[CAP];
+  __shared__ int offsets[CAP_PAD];
   __shared__ int scratch[40];
   int len[NNZ_PER_THREAD];
 #pragma unroll
@@ -516,26 +516,25 @@ __global__ void k_debug_sort_compact(const int32_t* rows, const int32_t* cols, c
   for (int p = tid; p < CAP; p += THREADS) {
     if (p < n) {
       const uint64_t key = ((uint64_t)(rows[p] - rmin) << colbits) | (uint64_t)(cols[p] - cmin);
-      S.words[p] = (key << IDXBITS) | (uint64_t)p;
+      S.words[pad32(p)] = (key << IDXBITS) | (uint64_t)p;
       S.vals[p] = vals[p];
     } else {
-      S.words[p] = ~0ull;
+      S.words[pad32(p)] = ~0ull;
     }
   }
   __syncthreads();
-  CElem<uint64_t, double> x[ITEMS];
-  sort_and_scan<uint64_t, double>(S, n, rowbits + colbits, colbits, x);
+  uint64_t k[ITEMS];
+  double ev[ITEMS];
+  load_and_sort<uint64_t, double>(S, rowbits + colbits, k);
+  const ScanCtx<uint64_t, double> ctx = compaction_prepare<uint64_t, double>(S, k, n, colbits, ev);
   const uint64_t colmask = colbits ? ((1ull << colbits) - 1) : 0;
-#pragma unroll
-  for (int i = 0; i < ITEMS; ++i) {
-    const int idx = tid * ITEMS + i;
-    if (idx < n) {
-      orow[idx] = rmin + (int)(x[i].key >> colbits);
-      ocol[idx] = cmin + (int)(x[i].key & colmask);
-      oval[idx] = x[i].val;
-      ostate[idx] = x[i].state;
-    }
-  }
+  compaction_emit<uint64_t, double>(k, ev, n, colbits, ctx,
+                                    [&](int idx, uint64_t key, double val, uint32_t state, bool, bool) {
+    orow[idx] = rmin + (int)(key >> colbits);
+    ocol[idx] = cmin + (int)(key & colmask);
+    oval[idx] = val;
+    ostate[idx] = state;
+  });
 }
 
 template <typename P>
