@@ -72,6 +72,7 @@ __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 // receives the block sum.  Contains two __syncthreads().
 template <typename V>
 __device__ __forceinline__ V block_exclusive_sum(V x, V* scratch, V* total) {
+  constexpr int NW = THREADS / 32;
   const int lane = lane_id(), w = warp_id();
   V inc = x;
 #pragma unroll
@@ -81,16 +82,18 @@ __device__ __forceinline__ V block_exclusive_sum(V x, V* scratch, V* total) {
   }
   if (lane == 31) scratch[w] = inc;
   __syncthreads();
-  if (threadIdx.x == 0) {
-    V run = 0;
-    for (int i = 0; i < THREADS / 32; ++i) { V t = scratch[i]; scratch[i] = run; run += t; }
-    scratch[THREADS / 32] = run;
+  // every warp scans the NW warp totals in its low lanes (no serial loop)
+  V t = lane < NW ? scratch[lane] : (V)0;
+  V ti = t;
+#pragma unroll
+  for (int d = 1; d < NW; d <<= 1) {
+    V y = __shfl_up_sync(0xffffffffu, ti, d);
+    if (lane >= d) ti += y;
   }
-  __syncthreads();
-  V res = scratch[w] + inc - x;
-  *total = scratch[THREADS / 32];
+  const V wpre = __shfl_sync(0xffffffffu, ti - t, w);
+  *total = __shfl_sync(0xffffffffu, ti, NW - 1);
   __syncthreads();          // scratch may be reused by the caller right away
-  return res;
+  return wpre + inc - x;
 }
 
 // Block-wide inclusive max scan (one value per thread).  Two __syncthreads().
@@ -116,6 +119,7 @@ __device__ __forceinline__ int block_inclusive_max(int x, int* scratch) {
 
 // Block-wide exclusive max scan (identity 0, the "clear(Offsets)" value of Alg. 2).
 __device__ __forceinline__ int block_exclusive_max(int x, int* scratch) {
+  constexpr int NW = THREADS / 32;
   const int lane = lane_id(), w = warp_id();
   int inc = x;
 #pragma unroll
@@ -127,33 +131,36 @@ __device__ __forceinline__ int block_exclusive_max(int x, int* scratch) {
   if (lane == 0) ex = 0;
   if (lane == 31) scratch[w] = inc;
   __syncthreads();
-  if (threadIdx.x == 0) {
-    int run = 0;
-    for (int i = 0; i < THREADS / 32; ++i) { int t = scratch[i]; scratch[i] = run; run = max(run, t); }
+  int t = lane < NW ? scratch[lane] : 0;
+#pragma unroll
+  for (int d = 1; d < NW; d <<= 1) {
+    int y = __shfl_up_sync(0xffffffffu, t, d);
+    if (lane >= d) t = max(t, y);
   }
+  int wpre = __shfl_up_sync(0xffffffffu, t, 1);
+  wpre = __shfl_sync(0xffffffffu, lane == 0 ? 0 : wpre, w);
   __syncthreads();
-  int res = max(scratch[w], ex);
-  __syncthreads();
-  return res;
+  return max(wpre, ex);
 }
 
 // Block-wide min/max reduction of four ints (rmin, rmax, cmin, cmax).
 __device__ __forceinline__ void block_minmax4(int& a_min, int& a_max, int& b_min, int& b_max, int* scratch) {
+  constexpr int NW = THREADS / 32;
   a_min = __reduce_min_sync(0xffffffffu, a_min);
   a_max = __reduce_max_sync(0xffffffffu, a_max);
   b_min = __reduce_min_sync(0xffffffffu, b_min);
   b_max = __reduce_max_sync(0xffffffffu, b_max);
-  const int w = warp_id();
-  if (lane_id() == 0) {
+  const int w = warp_id(), lane = lane_id();
+  if (lane == 0) {
     scratch[4 * w + 0] = a_min; scratch[4 * w + 1] = a_max;
     scratch[4 * w + 2] = b_min; scratch[4 * w + 3] = b_max;
   }
   __syncthreads();
-  a_min = scratch[0]; a_max = scratch[1]; b_min = scratch[2]; b_max = scratch[3];
-  for (int i = 1; i < THREADS / 32; ++i) {
-    a_min = min(a_min, scratch[4 * i + 0]); a_max = max(a_max, scratch[4 * i + 1]);
-    b_min = min(b_min, scratch[4 * i + 2]); b_max = max(b_max, scratch[4 * i + 3]);
-  }
+  const int q = lane < NW ? lane : 0;
+  a_min = __reduce_min_sync(0xffffffffu, scratch[4 * q + 0]);
+  a_max = __reduce_max_sync(0xffffffffu, scratch[4 * q + 1]);
+  b_min = __reduce_min_sync(0xffffffffu, scratch[4 * q + 2]);
+  b_max = __reduce_max_sync(0xffffffffu, scratch[4 * q + 3]);
   __syncthreads();
 }
 

@@ -71,23 +71,32 @@ __device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, E
   T ev[ITEMS];
   load_and_sort<Word, T>(S.s, rowbits + colbits, k);
   const ScanCtx<Word, T> ctx = compaction_prepare<Word, T>(S.s, k, n, colbits, ev);
-  const int total = st_count(ctx.total.state);
-  const int rc_last = st_row_count(ctx.total.state);
-  const int lastrel = (int)(ctx.total.key >> colbits);
+  int* stage_col = reinterpret_cast<int*>(S.s.words);
+  T* stage_val = S.s.vals;
+  int* misc = S.s.misc;
+  // element n-1 (the last valid one) ends the last run and row: its state gives the
+  // compacted total and the last row's count; publish it first
+  const int owner = (n - 1) / ITEMS;
+  if (threadIdx.x == owner) {
+    compaction_emit<Word, T>(k, ev, n, colbits, ctx, [&](int idx, Word key, T, uint32_t state, bool) {
+      if (idx == n - 1) {
+        misc[0] = st_count(state);
+        misc[1] = st_row_count(state);
+        misc[2] = (int)(key >> colbits);
+      }
+    });
+  }
+  __syncthreads();   // also: every read of the sort buffers is done, staging may start
+  const int total = misc[0], rc_last = misc[1], lastrel = misc[2];
   // keep the last row for the next iteration (L366) unless the block is done or the
   // row no longer fits the kept budget (reading R13: then it is written as a partial
   // chunk and merged later)
   const bool keep = size_after > 0 && rc_last <= KEEP;
   const int nchunk = total - (keep ? rc_last : 0);
-  int* stage_col = reinterpret_cast<int*>(S.s.words);
-  T* stage_val = S.s.vals;
-  int* misc = S.s.misc;
   const Word colmask = colbits ? (((Word)1 << colbits) - (Word)1) : (Word)0;
   // compacted element p goes to staging slot p: [0, nchunk) is the chunk, the kept
   // row stays at [nchunk, total) for the next iteration
-  compaction_emit<Word, T>(k, ev, n, colbits, ctx, [&](int, Word key, T val, uint32_t state, bool run_end,
-                                                       bool row_end) {
-    if (!run_end) return;
+  compaction_emit<Word, T>(k, ev, n, colbits, ctx, [&](int, Word key, T val, uint32_t state, bool row_end) {
     const int p = st_count(state) - 1;
     stage_col[p] = cmin + (int)(key & colmask);
     stage_val[p] = val;
@@ -266,7 +275,7 @@ __global__ void __launch_bounds__(THREADS, 3) k_esc(EscArgs a) {
     // dynamic bit reduction (L342-L344): only the row and column ranges present
     const int rowbits = bit_width_u64((uint64_t)(rmax - rmin));
     const int colbits = bit_width_u64((uint64_t)((int64_t)cmax - (int64_t)cmin));
-    if (rowbits + colbits + IDXBITS <= 32)
+    if (rowbits + colbits + IDXBITS < 32)
       esc_iteration<uint32_t, T>(S, a, st, consume, size_after, ares, col, kc, rmin, cmin, rowbits, colbits,
                                  pool_base, desc_base);
     else

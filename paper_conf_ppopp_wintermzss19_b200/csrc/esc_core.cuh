@@ -153,13 +153,15 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
     }
     if (lane == 31) s_warp[w] = inc;
     __syncthreads();
-    uint32_t wpre = 0, grand = 0;
+    uint32_t wt = lane < THREADS / 32 ? s_warp[lane] : 0u;
 #pragma unroll
-    for (int q = 0; q < THREADS / 32; ++q) {
-      const uint32_t t = s_warp[q];
-      wpre += q < w ? t : 0u;
-      grand += t;
+    for (int d = 1; d < THREADS / 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, wt, d);
+      if (lane >= d) wt += y;
     }
+    const uint32_t grand = __shfl_sync(0xffffffffu, wt, THREADS / 32 - 1);
+    uint32_t wpre = __shfl_up_sync(0xffffffffu, wt, 1);
+    wpre = __shfl_sync(0xffffffffu, lane == 0 ? 0u : wpre, w);
     // digits 16..31 (high halves) follow all of 0..15 (low halves)
     uint32_t run = wpre + inc - sum + ((grand & 0xFFFFu) << 16);
 #pragma unroll
@@ -238,8 +240,8 @@ struct SortSmem {
                                       // half); after the sort: int32 staging of output
                                       // columns at plain index p
   T vals[CAP];                        // values by position; after the sort: output staging
-  CElem<uint64_t, T> warp_agg[THREADS / 32];
-  uint8_t warp_has[THREADS / 32];
+  CElem<uint64_t, T> warp_agg[2 * (THREADS / 32) + 1];
+  uint8_t warp_has[2 * (THREADS / 32) + 1];
   uint32_t swarp[THREADS / 32];
   int scratch[40];
   int misc[16];
@@ -247,26 +249,25 @@ struct SortSmem {
 
 // The compaction scan (Alg. 3) over the sorted words of a thread (blocked layout).
 // Within a thread the scan is a left fold; because the input is sorted, applying the
-// CombineScanOperator to a running element and the next item only needs the previous
-// item's run-end / row-end flags (a.key == b.key  <=>  previous item is not a run end;
-// equalRow  <=>  previous item is not a row end).  Across threads the operator itself
+// CombineScanOperator to the running element and the next item only needs to know
+// whether the previous item ended a run / a row (a.key == b.key  <=>  no run end
+// between them; equalRow  <=>  no row end).  Across threads the operator itself
 // combines the per-thread aggregates (warp Kogge-Stone, then the warps in order).
-//   prepare: flags, values (into registers), the thread aggregate, the block scan of the
-//            aggregates; returns the carry-in and the block total (element n-1).
+// Padding words (all ones) sort after the n valid elements and carry a key larger than
+// every valid key (callers guarantee keybits + IDXBITS < word width), so they only form
+// trailing runs of their own and never change a valid element's scan result; no
+// per-item validity predicates are needed.
+//   prepare: values into registers, the thread aggregate, the block scan of the
+//            aggregates; returns the carry-in and publishes element n-1's scan result.
 //   emit:    re-folds the thread's items from the carry and calls
-//            f(idx, key, value, state, run_end, row_end) for every valid element.
+//            f(idx, key, value, state, row_end) at every run end with idx < n.
 // The tree is fixed by (THREADS, ITEMS): results are bit-stable run to run.
 template <typename Word, typename T>
 struct ScanCtx {
   CElem<Word, T> carry;
   bool has_carry;
-  CElem<Word, T> total;
-  uint32_t flags;        // bit 2i: run end of item i, bit 2i+1: row end
+  Word next_last;        // key following this thread's last item
 };
-
-__device__ __forceinline__ uint32_t init_state(bool run_end, bool row_end) {
-  return row_end ? ST_END_ROW : (run_end ? ST_END_COMP : 0u);
-}
 
 template <typename Word, typename T>
 __device__ __forceinline__ ScanCtx<Word, T> compaction_prepare(SortSmem<T>& s, const Word (&k)[ITEMS], int n,
@@ -276,108 +277,89 @@ __device__ __forceinline__ ScanCtx<Word, T> compaction_prepare(SortSmem<T>& s, c
   const Word posmask = (Word)(CAP - 1);
   const int base = threadIdx.x * ITEMS;
   ScanCtx<Word, T> ctx;
-  uint32_t flags = 0;
-  T val = (T)0;
+  ctx.next_last = (base + ITEMS < CAP) ? (sw[pad32(base + ITEMS)] >> IDXBITS) : ~(Word)0;
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) ev[i] = s.vals[(int)(k[i] & posmask)];
+  // thread-local fold (state bits: see Alg. 3)
+  T val = ev[0];
   uint32_t state = 0;
 #pragma unroll
   for (int i = 0; i < ITEMS; ++i) {
-    const int idx = base + i;
     const Word key = k[i] >> IDXBITS;
-    Word nkey;
-    if (i + 1 < ITEMS) nkey = k[i + 1] >> IDXBITS;
-    else nkey = (idx + 1 < CAP) ? (sw[pad32(idx + 1)] >> IDXBITS) : key;
-    const bool last = idx >= n - 1;
-    const bool run_end = last || nkey != key;
-    const bool row_end = last || (nkey >> colbits) != (key >> colbits);
-    flags |= ((uint32_t)run_end << (2 * i)) | ((uint32_t)row_end << (2 * i + 1));
-    ev[i] = idx < n ? s.vals[(int)(k[i] & posmask)] : (T)0;
-    if (i == 0) {
-      val = ev[0];
-      state = init_state(run_end, row_end);
-    } else if (idx < n) {
-      const bool prun = (flags >> (2 * i - 2)) & 1u, prow = (flags >> (2 * i - 1)) & 1u;
-      val = prun ? ev[i] : val + ev[i];
-      state = (prow ? (state & 0x0000FFFEu) : (state & 0xFFFEFFFEu)) + init_state(run_end, row_end);
+    const Word nkey = (i + 1 < ITEMS) ? (k[i + 1] >> IDXBITS) : ctx.next_last;
+    const bool run_end = nkey != key;
+    const bool row_end = (nkey >> colbits) != (key >> colbits);
+    const uint32_t st0 = row_end ? ST_END_ROW : (run_end ? ST_END_COMP : 0u);
+    if (i > 0) {
+      const Word pkey = k[i - 1] >> IDXBITS;
+      val = pkey != key ? ev[i] : val + ev[i];
+      state = ((pkey >> colbits) != (key >> colbits) ? (state & 0x0000FFFEu) : (state & 0xFFFEFFFEu)) + st0;
+    } else {
+      state = st0;
     }
   }
-  ctx.flags = flags;
-  const bool has = base < n;
-  CElem<Word, T> agg;
-  agg.key = k[min(ITEMS - 1, max(0, n - 1 - base))] >> IDXBITS;
-  agg.val = val;
-  agg.state = state;
-  // warp inclusive scan of (has, agg)
-  CElem<Word, T> inc = agg;
-  bool hinc = has;
+  CElem<Word, T> inc;
+  inc.key = k[ITEMS - 1] >> IDXBITS;
+  inc.val = val;
+  inc.state = state;
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
-    CElem<Word, T> y = shfl_up_elem(inc, d);
-    const bool hy = __shfl_up_sync(0xffffffffu, (int)hinc, d) != 0;
-    if (lane >= d && hy) {
-      inc = hinc ? combine_op(y, inc, colbits) : y;
-      hinc = true;
-    }
+    const CElem<Word, T> y = shfl_up_elem(inc, d);
+    if (lane >= d) inc = combine_op(y, inc, colbits);
   }
-  CElem<Word, T> ex = shfl_up_elem(inc, 1);
-  const bool hex = __shfl_up_sync(0xffffffffu, (int)hinc, 1) != 0 && lane > 0;
+  const CElem<Word, T> ex = shfl_up_elem(inc, 1);
   CElem<Word, T>* wagg = reinterpret_cast<CElem<Word, T>*>(s.warp_agg);
-  if (lane == 31) {
-    wagg[w] = inc;
-    s.warp_has[w] = hinc;
-  }
+  if (lane == 31) wagg[w] = inc;
   __syncthreads();
-  CElem<Word, T> wp, tot;
-  bool hwp = false, htot = false;
-#pragma unroll
-  for (int q = 0; q < THREADS / 32; ++q) {
-    if (s.warp_has[q]) {
-      const CElem<Word, T> v = wagg[q];
-      if (q < w) { wp = hwp ? combine_op(wp, v, colbits) : v; hwp = true; }
-      tot = htot ? combine_op(tot, v, colbits) : v;
-      htot = true;
+  // one thread turns the warp aggregates into inclusive warp prefixes (fixed order)
+  if (threadIdx.x == 0) {
+    CElem<Word, T> run = wagg[0];
+    for (int q = 1; q < THREADS / 32; ++q) {
+      run = combine_op(run, wagg[q], colbits);
+      wagg[q] = run;
     }
   }
-  if (hwp && hex) { ctx.carry = combine_op(wp, ex, colbits); ctx.has_carry = true; }
-  else if (hwp) { ctx.carry = wp; ctx.has_carry = true; }
-  else if (hex) { ctx.carry = ex; ctx.has_carry = true; }
-  else { ctx.has_carry = false; }
-  ctx.total = tot;
   __syncthreads();
+  if (w > 0) {
+    const CElem<Word, T> wp = wagg[w - 1];
+    ctx.carry = lane > 0 ? combine_op(wp, ex, colbits) : wp;
+    ctx.has_carry = true;
+  } else {
+    ctx.carry = ex;
+    ctx.has_carry = lane > 0;
+  }
   return ctx;
 }
 
-// (prepare ends with a barrier: after it the sort buffers may be overwritten)
-template <typename Word, typename T, typename F>
+template <typename Word, typename T, bool ALL = false, typename F>
 __device__ __forceinline__ void compaction_emit(const Word (&k)[ITEMS], const T (&ev)[ITEMS], int n, int colbits,
                                                 const ScanCtx<Word, T>& ctx, F&& f) {
   const int base = threadIdx.x * ITEMS;
-  T val = (T)0;
-  uint32_t state = 0;
+  T val;
+  uint32_t state;
+  Word pkey;
+  if (ctx.has_carry) {
+    val = ctx.carry.val;
+    state = ctx.carry.state;
+    pkey = ctx.carry.key;
+  }
 #pragma unroll
   for (int i = 0; i < ITEMS; ++i) {
-    const int idx = base + i;
-    if (idx < n) {
-      const Word key = k[i] >> IDXBITS;
-      const bool run_end = (ctx.flags >> (2 * i)) & 1u;
-      const bool row_end = (ctx.flags >> (2 * i + 1)) & 1u;
-      const uint32_t st0 = init_state(run_end, row_end);
-      if (i == 0) {
-        if (ctx.has_carry) {
-          const bool eq_key = ctx.carry.key == key;
-          const bool eq_row = (ctx.carry.key >> colbits) == (key >> colbits);
-          val = eq_key ? ctx.carry.val + ev[0] : ev[0];
-          state = (eq_row ? (ctx.carry.state & 0xFFFEFFFEu) : (ctx.carry.state & 0x0000FFFEu)) + st0;
-        } else {
-          val = ev[0];
-          state = st0;
-        }
-      } else {
-        const bool prun = (ctx.flags >> (2 * i - 2)) & 1u, prow = (ctx.flags >> (2 * i - 1)) & 1u;
-        val = prun ? ev[i] : val + ev[i];
-        state = (prow ? (state & 0x0000FFFEu) : (state & 0xFFFEFFFEu)) + st0;
-      }
-      f(idx, key, val, state, run_end, row_end);
+    const Word key = k[i] >> IDXBITS;
+    const Word nkey = (i + 1 < ITEMS) ? (k[i + 1] >> IDXBITS) : ctx.next_last;
+    const bool run_end = nkey != key;
+    const bool row_end = (nkey >> colbits) != (key >> colbits);
+    const uint32_t st0 = row_end ? ST_END_ROW : (run_end ? ST_END_COMP : 0u);
+    if (i > 0 || ctx.has_carry) {
+      val = pkey != key ? ev[i] : val + ev[i];
+      state = ((pkey >> colbits) != (key >> colbits) ? (state & 0x0000FFFEu) : (state & 0xFFFEFFFEu)) + st0;
+    } else {
+      val = ev[0];
+      state = st0;
     }
+    pkey = key;
+    const int idx = base + i;
+    if ((ALL || run_end) && idx < n) f(idx, key, val, state, row_end);
   }
 }
 

@@ -528,8 +528,8 @@ __global__ void k_debug_sort_compact(const int32_t* rows, const int32_t* cols, c
   load_and_sort<uint64_t, double>(S, rowbits + colbits, k);
   const ScanCtx<uint64_t, double> ctx = compaction_prepare<uint64_t, double>(S, k, n, colbits, ev);
   const uint64_t colmask = colbits ? ((1ull << colbits) - 1) : 0;
-  compaction_emit<uint64_t, double>(k, ev, n, colbits, ctx,
-                                    [&](int idx, uint64_t key, double val, uint32_t state, bool, bool) {
+  compaction_emit<uint64_t, double, true>(k, ev, n, colbits, ctx,
+                                          [&](int idx, uint64_t key, double val, uint32_t state, bool) {
     orow[idx] = rmin + (int)(key >> colbits);
     ocol[idx] = cmin + (int)(key & colmask);
     oval[idx] = val;
