@@ -5,22 +5,35 @@
 // A chunk's rows are contiguous in its data and, apart from a shared first / last
 // row (supplied by the merged copy, L428), contiguous in C as well, so every chunk is
 // a single contiguous copy.  Shared rows copy their merged data from the merge pool.
+// B200: one warp per chunk (chunks average a few hundred elements), streaming
+// (evict-first) loads and stores since neither side is re-read.
 #include "kernels.cuh"
 
 namespace acs {
 
+// One warp per chunk (or shared row): 4 independent element loads per lane in flight.
 template <typename T>
-__device__ __forceinline__ void block_copy(const int32_t* __restrict__ scol, const T* __restrict__ sval,
-                                           int32_t* __restrict__ dcol, T* __restrict__ dval, int n) {
-  for (int i = threadIdx.x; i < n; i += blockDim.x) {
-    dcol[i] = scol[i];
-    dval[i] = sval[i];
+__device__ __forceinline__ void warp_copy(const int32_t* __restrict__ scol, const T* __restrict__ sval,
+                                          int32_t* __restrict__ dcol, T* __restrict__ dval, int n, int lane) {
+  int i = lane;
+  for (; i + 96 < n; i += 128) {
+    const int32_t c0 = __ldcs(scol + i), c1 = __ldcs(scol + i + 32), c2 = __ldcs(scol + i + 64), c3 = __ldcs(scol + i + 96);
+    const T v0 = __ldcs(sval + i), v1 = __ldcs(sval + i + 32), v2 = __ldcs(sval + i + 64), v3 = __ldcs(sval + i + 96);
+    __stcs(dcol + i, c0); __stcs(dcol + i + 32, c1); __stcs(dcol + i + 64, c2); __stcs(dcol + i + 96, c3);
+    __stcs(dval + i, v0); __stcs(dval + i + 32, v1); __stcs(dval + i + 64, v2); __stcs(dval + i + 96, v3);
+  }
+  for (; i < n; i += 32) {
+    __stcs(dcol + i, __ldcs(scol + i));
+    __stcs(dval + i, __ldcs(sval + i));
   }
 }
 
+constexpr int COPY_WARPS = 8;
+
 template <typename T>
-__global__ void __launch_bounds__(256) k_copy(CopyArgs a) {
-  const int64_t x = blockIdx.x;
+__global__ void __launch_bounds__(32 * COPY_WARPS) k_copy(CopyArgs a) {
+  const int64_t x = (int64_t)blockIdx.x * COPY_WARPS + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
   if (x < a.max_chunks) {
     if (x >= *a.total_chunks_dev) return;
     const ChunkDesc d = a.dense[x];
@@ -29,23 +42,24 @@ __global__ void __launch_bounds__(256) k_copy(CopyArgs a) {
     if (s >= e) return;
     const int dst_row = (d.flags & 1) ? d.first_row + 1 : d.first_row;
     const int64_t dst = a.row_ptr[dst_row];
-    block_copy<T>(a.pool_col + d.data_off + s, reinterpret_cast<const T*>(a.pool_val) + d.data_off + s,
-                  a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, e - s);
+    warp_copy<T>(a.pool_col + d.data_off + s, reinterpret_cast<const T*>(a.pool_val) + d.data_off + s,
+                 a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, e - s, lane);
   } else {
     const int64_t i = x - a.max_chunks;
     if (i >= a.nshared) return;
     const SharedRow sh = a.shared[i];
     const int64_t dst = a.row_ptr[sh.row];
-    block_copy<T>(a.merge_col + sh.merge_off, reinterpret_cast<const T*>(a.merge_val) + sh.merge_off,
-                  a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, sh.merged);
+    warp_copy<T>(a.merge_col + sh.merge_off, reinterpret_cast<const T*>(a.merge_val) + sh.merge_off,
+                 a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, sh.merged, lane);
   }
 }
 
 void launch_copy(const CopyArgs& a, bool f64, cudaStream_t st) {
-  const int64_t grid = a.max_chunks + a.nshared;
-  if (grid <= 0) return;
-  if (f64) k_copy<double><<<(unsigned)grid, 256, 0, st>>>(a);
-  else k_copy<float><<<(unsigned)grid, 256, 0, st>>>(a);
+  const int64_t items = a.max_chunks + a.nshared;
+  if (items <= 0) return;
+  const unsigned grid = (unsigned)((items + COPY_WARPS - 1) / COPY_WARPS);
+  if (f64) k_copy<double><<<grid, 32 * COPY_WARPS, 0, st>>>(a);
+  else k_copy<float><<<grid, 32 * COPY_WARPS, 0, st>>>(a);
 }
 
 }  // namespace acs

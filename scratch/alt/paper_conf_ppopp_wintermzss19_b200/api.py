@@ -1,0 +1,276 @@
+"""Python binding of the AC-SpGEMM C ABI (argument marshalling only).
+
+torch supplies device memory and streams; every step of C = A·B runs in the CUDA
+kernels of libacspgemm.so.  Names follow include/acspgemm.h.
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+from typing import Optional, Sequence
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import CsrIn, CsrOut, Info, Options, check, load
+
+F32, F64 = 0, 1
+STAGES = ("GLB", "ESC", "MCC", "MM", "PM", "SM", "SCAN", "CC")
+
+
+@dataclass
+class DeviceCSR:
+    """CSR matrix in CUDA memory: row_ptr/col int32, val float32 or float64."""
+    rows: int
+    cols: int
+    row_ptr: torch.Tensor
+    col: torch.Tensor
+    val: torch.Tensor
+
+    @property
+    def nnz(self) -> int:
+        return int(self.col.numel())
+
+    @property
+    def dtype(self):
+        return self.val.dtype
+
+    @staticmethod
+    def from_numpy(rows, cols, row_ptr, col, val, device="cuda", dtype=None) -> "DeviceCSR":
+        v = np.asarray(val)
+        if dtype is not None:
+            v = v.astype(dtype)
+        return DeviceCSR(int(rows), int(cols),
+                         torch.from_numpy(np.ascontiguousarray(row_ptr, dtype=np.int32)).to(device),
+                         torch.from_numpy(np.ascontiguousarray(col, dtype=np.int32)).to(device),
+                         torch.from_numpy(np.ascontiguousarray(v)).to(device))
+
+    @staticmethod
+    def from_host(M, device="cuda", dtype=None) -> "DeviceCSR":
+        """From any object with rows, cols, row_ptr, col, val numpy arrays."""
+        return DeviceCSR.from_numpy(M.rows, M.cols, M.row_ptr, M.col, M.val, device, dtype)
+
+    def to_numpy(self):
+        return (self.row_ptr.cpu().numpy(), self.col.cpu().numpy(), self.val.cpu().numpy())
+
+
+def _dtype_code(t: torch.dtype) -> int:
+    if t == torch.float64:
+        return F64
+    if t == torch.float32:
+        return F32
+    raise TypeError(f"unsupported value dtype {t} (float32/float64)")
+
+
+def _csr_in(M: DeviceCSR, row_ptr: Optional[torch.Tensor] = None, rows: Optional[int] = None,
+            nnz: Optional[int] = None) -> CsrIn:
+    rp = M.row_ptr if row_ptr is None else row_ptr
+    for t in (rp, M.col, M.val):
+        if not t.is_cuda or not t.is_contiguous():
+            raise ValueError("DeviceCSR tensors must be contiguous CUDA tensors")
+    if rp.dtype != torch.int32 or M.col.dtype != torch.int32:
+        raise TypeError("row_ptr / col must be int32")
+    r = M.rows if rows is None else rows
+    n = M.nnz if nnz is None else nnz
+    return CsrIn(r, M.cols, n, rp.data_ptr(), M.col.data_ptr(), M.val.data_ptr())
+
+
+def _stream_ptr(stream: Optional[torch.cuda.Stream]) -> ctypes.c_void_p:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+class Plan:
+    """A reusable multiply plan (owns the chunk pool and helper memory)."""
+
+    def __init__(self, pool_limit_bytes: int = 0, validate: bool = False, stage_times: bool = False,
+                 num_segments: int = 8):
+        lib = load()
+        opt = Options()
+        lib.acspgemm_options_default(ctypes.byref(opt))
+        opt.pool_limit_bytes = int(pool_limit_bytes)
+        opt.validate_inputs = int(bool(validate))
+        opt.collect_stage_times = int(bool(stage_times))
+        opt.num_segments = int(num_segments)
+        h = ctypes.c_void_p()
+        check(lib.acspgemm_plan_create(ctypes.byref(h), ctypes.byref(opt)), "acspgemm_plan_create")
+        self._h = h
+        self._lib = lib
+        self._dtype = None
+        self._rows = 0
+        self._cols = 0
+
+    def close(self) -> None:
+        if getattr(self, "_h", None) is not None and self._h.value:
+            self._lib.acspgemm_plan_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def set_segments(self, rows: Optional[Sequence[int]]) -> None:
+        if rows is None:
+            check(self._lib.acspgemm_set_segments(self._h, 0, None), "acspgemm_set_segments")
+            return
+        arr = (ctypes.c_int64 * len(rows))(*[int(r) for r in rows])
+        check(self._lib.acspgemm_set_segments(self._h, len(rows) - 1, arr), "acspgemm_set_segments")
+
+    def symbolic(self, A: DeviceCSR, B: DeviceCSR, stream=None, A_view=None) -> int:
+        if A.dtype != B.dtype:
+            raise TypeError("A and B must have the same value dtype")
+        a = _csr_in(A) if A_view is None else A_view
+        b = _csr_in(B)
+        nnz = ctypes.c_int64(0)
+        check(self._lib.acspgemm_symbolic(self._h, ctypes.byref(a), ctypes.byref(b), _dtype_code(A.dtype),
+                                          _stream_ptr(stream), ctypes.byref(nnz)), "acspgemm_symbolic")
+        self._dtype = A.dtype
+        self._rows = a.rows
+        self._cols = B.cols
+        return int(nnz.value)
+
+    def numeric(self, row_ptr: torch.Tensor, col: torch.Tensor, val: torch.Tensor, stream=None) -> None:
+        c = CsrOut(0, 0, 0, row_ptr.data_ptr(), col.data_ptr(), val.data_ptr())
+        check(self._lib.acspgemm_numeric(self._h, ctypes.byref(c), _stream_ptr(stream)), "acspgemm_numeric")
+
+    def multiply(self, A: DeviceCSR, B: DeviceCSR, stream=None, A_view=None) -> DeviceCSR:
+        """symbolic -> allocate C with torch on the device -> numeric."""
+        nnz = self.symbolic(A, B, stream, A_view)
+        dev = A.val.device
+        rows = self._rows
+        rp = torch.empty(rows + 1, dtype=torch.int32, device=dev)
+        col = torch.empty(max(nnz, 1), dtype=torch.int32, device=dev)
+        val = torch.empty(max(nnz, 1), dtype=A.dtype, device=dev)
+        self.numeric(rp, col, val, stream)
+        return DeviceCSR(rows, B.cols, rp, col[:nnz], val[:nnz])
+
+    def info(self) -> dict:
+        inf = Info()
+        check(self._lib.acspgemm_plan_info(self._h, ctypes.byref(inf)), "acspgemm_plan_info")
+        d = {name: getattr(inf, name) for name, _ in Info._fields_ if name != "segment_rows"}
+        d["segment_rows"] = [inf.segment_rows[i] for i in range(inf.nsegments + 1)] if inf.nsegments else []
+        return d
+
+    def stage_times(self) -> dict:
+        buf = (ctypes.c_float * 8)()
+        check(self._lib.acspgemm_stage_times(self._h, buf, 8), "acspgemm_stage_times")
+        return {k: float(buf[i]) for i, k in enumerate(STAGES)}
+
+    def block_row_starts(self) -> np.ndarray:
+        n = self.info()["nblocks"]
+        out = np.zeros(max(n, 1), dtype=np.int32)
+        check(self._lib.acspgemm_block_row_starts(self._h, out.ctypes.data_as(_lib.PI32), n),
+              "acspgemm_block_row_starts")
+        return out[:n]
+
+
+def multiply(A: DeviceCSR, B: DeviceCSR, stream=None, **plan_kw) -> DeviceCSR:
+    """C = A·B with a temporary plan (two-phase API, C allocated by torch)."""
+    p = Plan(**plan_kw)
+    try:
+        return p.multiply(A, B, stream)
+    finally:
+        p.close()
+
+
+def multiply_lib_alloc(A: DeviceCSR, B: DeviceCSR, stream=None):
+    """C = A·B through acspgemm_multiply (the library allocates C with cudaMallocAsync).
+    Returns host numpy arrays (row_ptr, col, val) and frees the device C."""
+    lib = load()
+    a, b = _csr_in(A), _csr_in(B)
+    c = CsrOut()
+    st = _stream_ptr(stream)
+    check(lib.acspgemm_multiply(ctypes.byref(a), ctypes.byref(b), ctypes.byref(c), st, _dtype_code(A.dtype)),
+          "acspgemm_multiply")
+    try:
+        n = c.nnz
+        rp = np.empty(c.rows + 1, dtype=np.int32)
+        col = np.empty(n, dtype=np.int32)
+        val = np.empty(n, dtype=np.float64 if A.dtype == torch.float64 else np.float32)
+        torch.cuda.synchronize()
+        _memcpy_d2h(rp, c.row_ptr)
+        _memcpy_d2h(col, c.col_idx)
+        _memcpy_d2h(val, c.val)
+        return rp, col, val
+    finally:
+        check(lib.acspgemm_free_csr(ctypes.byref(c), st), "acspgemm_free_csr")
+        torch.cuda.synchronize()
+
+
+def _memcpy_d2h(dst: np.ndarray, src_ptr) -> None:
+    if dst.nbytes:
+        _cuda_memcpy(dst.ctypes.data, int(src_ptr), dst.nbytes)
+
+
+_cudart = None
+
+
+def _cuda_memcpy(dst: int, src: int, n: int) -> None:
+    global _cudart
+    if _cudart is None:
+        import glob
+        import os
+        cands = glob.glob(os.path.join(os.path.dirname(torch.__file__), "lib", "libcudart*.so*"))
+        cands += glob.glob("/usr/local/cuda/lib64/libcudart.so*")
+        _cudart = ctypes.CDLL(cands[0])
+        _cudart.cudaMemcpy.restype = ctypes.c_int
+        _cudart.cudaMemcpy.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int]
+    rc = _cudart.cudaMemcpy(ctypes.c_void_p(dst), ctypes.c_void_p(src), ctypes.c_size_t(n), 2)
+    if rc != 0:
+        raise RuntimeError(f"cudaMemcpy failed ({rc})")
+
+
+def canonical_segments(A: DeviceCSR, nseg: int = 8, stream=None) -> list:
+    lib = load()
+    a = _csr_in(A)
+    out = (ctypes.c_int64 * (nseg + 1))()
+    check(lib.acspgemm_canonical_segments(ctypes.byref(a), nseg, out, _stream_ptr(stream)),
+          "acspgemm_canonical_segments")
+    return [int(out[i]) for i in range(nseg + 1)]
+
+
+def pool_estimate_bytes(nA, nnzA, nB, mB, nnzB, value_bytes) -> float:
+    return float(load().acspgemm_pool_estimate_bytes(nA, nnzA, nB, mB, nnzB, value_bytes))
+
+
+def const(name: str) -> int:
+    ids = {"NPB": 0, "THREADS": 1, "ITEMS": 2, "CAP": 3, "KEEP": 4, "RADIX_BITS": 5, "SEGMENTS": 6,
+           "PATH_MAX_CHUNKS": 7}
+    return int(load().acspgemm_const(ids[name]))
+
+
+def debug_work_distribution(lengths: Sequence[int], draws: Sequence[int]):
+    """Alg. 2 on the GPU (one CTA): returns (ares, bres, remaining[ndraws, nentries])."""
+    lib = load()
+    L = np.ascontiguousarray(lengths, dtype=np.int32)
+    D = np.ascontiguousarray(draws, dtype=np.int32)
+    tot = int(D.sum())
+    ares = np.zeros(max(tot, 1), np.int32)
+    bres = np.zeros(max(tot, 1), np.int32)
+    rem = np.zeros(max(len(L) * len(D), 1), np.int32)
+    check(lib.acspgemm_debug_work_distribution(L.ctypes.data_as(_lib.PI32), len(L), D.ctypes.data_as(_lib.PI32),
+                                               len(D), ares.ctypes.data_as(_lib.PI32),
+                                               bres.ctypes.data_as(_lib.PI32), rem.ctypes.data_as(_lib.PI32)),
+          "acspgemm_debug_work_distribution")
+    return ares[:tot], bres[:tot], rem[:len(L) * len(D)].reshape(len(D), len(L))
+
+
+def debug_sort_compact(rows, cols, vals):
+    """Block radix sort + Alg. 3 compaction scan on the GPU (one CTA, n <= CAP)."""
+    lib = load()
+    r = np.ascontiguousarray(rows, dtype=np.int32)
+    c = np.ascontiguousarray(cols, dtype=np.int32)
+    v = np.ascontiguousarray(vals, dtype=np.float64)
+    n = len(r)
+    orow, ocol = np.zeros(max(n, 1), np.int32), np.zeros(max(n, 1), np.int32)
+    oval, ost = np.zeros(max(n, 1), np.float64), np.zeros(max(n, 1), np.uint32)
+    dp = ctypes.POINTER(ctypes.c_double)
+    check(lib.acspgemm_debug_sort_compact(r.ctypes.data_as(_lib.PI32), c.ctypes.data_as(_lib.PI32),
+                                          v.ctypes.data_as(dp), n, orow.ctypes.data_as(_lib.PI32),
+                                          ocol.ctypes.data_as(_lib.PI32), oval.ctypes.data_as(dp),
+                                          ost.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32))),
+          "acspgemm_debug_sort_compact")
+    return orow[:n], ocol[:n], oval[:n], ost[:n]

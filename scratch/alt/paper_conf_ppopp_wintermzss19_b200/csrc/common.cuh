@@ -12,10 +12,10 @@
 namespace acs {
 
 #ifndef ACS_THREADS
-#define ACS_THREADS 128
+#define ACS_THREADS 256
 #endif
 #ifndef ACS_ITEMS
-#define ACS_ITEMS 16
+#define ACS_ITEMS 8
 #endif
 #ifndef ESC_MIN_BLOCKS
 #define ESC_MIN_BLOCKS (ACS_THREADS == 256 ? 3 : 4)

@@ -1,0 +1,166 @@
+// Stage 1 — Global Load Balancing (§3.1, Alg. 1) plus the
+// per-block product bound used by the deterministic chunk allocator.
+//
+// A is split into canonical segments (nnz-balanced row ranges, reading
+// R21) and each segment into blocks of NPB consecutive nonzeros counted from the
+// segment's first nonzero ("splits the non-zeros of A uniformly, assigning the same
+// number to each thread block", L194).  Rows never straddle segments, so the block
+// decomposition -- and therefore every summation tree -- is the same whether the
+// segments run on one GPU or on several.
+#include "kernels.cuh"
+
+namespace acs {
+
+// seg layout: [0, MAX_SEGMENTS] rows | [MAX_SEGMENTS+1, ...] first nonzero | block base
+constexpr int SEG_STRIDE = MAX_SEGMENTS + 1;
+
+__global__ void k_segments(const int32_t* __restrict__ rp, int64_t rows, int nseg,
+                           const int64_t* __restrict__ explicit_rows, int64_t* __restrict__ seg,
+                           int32_t* __restrict__ nblocks) {
+  __shared__ int64_t s_rows[SEG_STRIDE], s_nz[SEG_STRIDE];
+  const int s = threadIdx.x;
+  const int64_t base = rp[0];
+  const int64_t nnz = (int64_t)rp[rows] - base;
+  if (s <= nseg) {
+    int64_t r;
+    if (explicit_rows) {
+      r = explicit_rows[s];
+    } else if (s == 0) {
+      r = 0;
+    } else if (s == nseg) {
+      r = rows;
+    } else {
+      // first row r with rp[r] - base >= ceil(s * nnz / nseg)
+      const int64_t target = (s * nnz + nseg - 1) / nseg;
+      int64_t lo = 0, hi = rows;
+      while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if ((int64_t)rp[mid] - base < target) lo = mid + 1; else hi = mid;
+      }
+      r = lo;
+    }
+    s_rows[s] = r;
+    s_nz[s] = rp[r];
+  }
+  __syncthreads();
+  if (s == 0) {
+    int64_t acc = 0;
+    for (int i = 0; i <= nseg; ++i) {
+      seg[i] = s_rows[i];
+      seg[SEG_STRIDE + i] = s_nz[i];
+      seg[2 * SEG_STRIDE + i] = acc;
+      if (i < nseg) acc += (s_nz[i + 1] - s_nz[i] + NPB - 1) / NPB;
+    }
+    *nblocks = (int32_t)acc;
+  }
+}
+
+void launch_segments(const CsrView& A, int nseg, const int64_t* explicit_rows, int64_t* seg,
+                     int32_t* nblocks_dev, cudaStream_t st) {
+  k_segments<<<1, 128, 0, st>>>(A.row_ptr, A.rows, nseg, explicit_rows, seg, nblocks_dev);
+}
+
+// Alg. 1: one thread per row of A.  Reading R4: rows with a == b are skipped.
+__global__ void k_glb(const int32_t* __restrict__ rp, int64_t rows, int nseg, const int64_t* __restrict__ seg,
+                      int32_t* __restrict__ block_row_starts) {
+  __shared__ int64_t s_rows[SEG_STRIDE], s_nz[SEG_STRIDE], s_base[SEG_STRIDE];
+  for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
+    s_rows[i] = seg[i];
+    s_nz[i] = seg[SEG_STRIDE + i];
+    s_base[i] = seg[2 * SEG_STRIDE + i];
+  }
+  __syncthreads();
+  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (tid >= rows) return;
+  const int64_t a0 = rp[tid], b0 = rp[tid + 1];
+  if (a0 == b0) return;
+  int s = 0;                                   // segment holding row tid
+  while (s + 1 < nseg && s_rows[s + 1] <= tid) ++s;
+  const int64_t a = a0 - s_nz[s], b = b0 - s_nz[s];
+  int64_t blocka = (a + NPB - 1) / NPB;        // divup(a, NNZ_PER_BLOCK)
+  const int64_t blockb = (b - 1) / NPB;        // (b - 1) / NNZ_PER_BLOCK
+  while (blocka <= blockb) {
+    block_row_starts[s_base[s] + blocka] = (int32_t)tid;
+    ++blocka;
+  }
+}
+
+void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* brs, int64_t max_blocks, cudaStream_t st) {
+  (void)max_blocks;
+  if (A.rows == 0) return;
+  const int T = 256;
+  k_glb<<<(unsigned)((A.rows + T - 1) / T), T, 0, st>>>(A.row_ptr, A.rows, nseg, seg, brs);
+}
+
+// Per block: nonzero range and the exact product count sum_p len(B_row(A.col[p])),
+// "inspecting B now comes with little additional cost" (L206).  One warp per block.
+// slots = ceil(products / (CAP - KEEP)) bounds the number of chunks the block emits
+// (every local ESC iteration consumes at least CAP - KEEP products and emits at most
+// one chunk), and products bounds its chunk elements (compaction never grows data).
+__global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* __restrict__ acol,
+                               const int32_t* __restrict__ brp, int nseg, const int64_t* __restrict__ seg,
+                               const int32_t* __restrict__ nblocks_dev, int64_t max_blocks,
+                               int32_t* __restrict__ nz_begin, int32_t* __restrict__ nz_end,
+                               int64_t* __restrict__ products, int64_t* __restrict__ slots) {
+  __shared__ int64_t s_nz[SEG_STRIDE], s_base[SEG_STRIDE];
+  for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
+    s_nz[i] = seg[SEG_STRIDE + i];
+    s_base[i] = seg[2 * SEG_STRIDE + i];
+  }
+  __syncthreads();
+  const int64_t b = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (b >= max_blocks) return;
+  const int nblocks = *nblocks_dev;
+  if (b >= nblocks) {
+    if (lane == 0) { products[b] = 0; slots[b] = 0; nz_begin[b] = 0; nz_end[b] = 0; }
+    return;
+  }
+  int s = 0;
+  while (s + 1 < nseg && s_base[s + 1] <= b) ++s;
+  const int64_t nzb = s_nz[s] + (b - s_base[s]) * NPB;
+  const int64_t nze = min(nzb + (int64_t)NPB, s_nz[s + 1]);
+  int64_t sum = 0;
+  for (int64_t p = nzb + lane; p < nze; p += 32) {
+    const int k = acol[p];
+    sum += brp[k + 1] - brp[k];
+  }
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, d);
+  if (lane == 0) {
+    products[b] = sum;
+    slots[b] = (sum + (CAP - KEEP) - 1) / (CAP - KEEP);
+    nz_begin[b] = (int32_t)nzb;
+    nz_end[b] = (int32_t)nze;
+  }
+}
+
+void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
+                         const int32_t* nblocks_dev, int64_t max_blocks, int32_t* nzb, int32_t* nze,
+                         int64_t* products, int64_t* slots, cudaStream_t st) {
+  if (max_blocks == 0) return;
+  const int T = 256, WPB = T / 32;
+  k_block_bounds<<<(unsigned)((max_blocks + WPB - 1) / WPB), T, 0, st>>>(
+      A.row_ptr, A.col, B.row_ptr, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots);
+}
+
+// Canonical-CSR check (reading R3): row_ptr monotone, columns strictly increasing and
+// in range.  Only run when acspgemm_options.validate_inputs is set.
+__global__ void k_validate(const int32_t* __restrict__ rp, const int32_t* __restrict__ col, int64_t rows,
+                           int64_t cols, int32_t* bad) {
+  const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= rows) return;
+  const int64_t a = rp[r], b = rp[r + 1];
+  if (b < a) { *bad = 1; return; }
+  for (int64_t p = a; p < b; ++p) {
+    const int c = col[p];
+    if (c < 0 || c >= cols || (p > a && col[p - 1] >= c)) { *bad = 1; return; }
+  }
+}
+
+void launch_validate(const CsrView& M, int32_t* bad, cudaStream_t st) {
+  if (M.rows == 0) return;
+  k_validate<<<(unsigned)((M.rows + 255) / 256), 256, 0, st>>>(M.row_ptr, M.col, M.rows, M.cols, bad);
+}
+
+}  // namespace acs

@@ -1,0 +1,131 @@
+// Internal host-side launchers of the AC-SpGEMM stage kernels (not part of the C ABI).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "common.cuh"
+
+namespace acs {
+
+struct CsrView {              // device CSR view; row_ptr values index col/val directly
+  int64_t rows, cols;
+  const int32_t* row_ptr;
+  const int32_t* col;
+  const void* val;
+};
+
+// ---- stage 1: global load balancing (glb.cu) ----------------------------------
+// seg_rows_host: explicit segment row boundaries (nseg+1) or nullptr for canonical.
+// Writes seg tables to `seg` (device, int64[4*(MAX_SEGMENTS+1)]): rows | nz | block base.
+void launch_segments(const CsrView& A, int nseg, const int64_t* seg_rows_dev_or_null,
+                     int64_t* seg, int32_t* nblocks_dev, cudaStream_t st);
+void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* block_row_starts,
+                int64_t max_blocks, cudaStream_t st);
+void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
+                         const int32_t* nblocks_dev, int64_t max_blocks, int32_t* blk_nz_begin,
+                         int32_t* blk_nz_end, int64_t* blk_products, int64_t* blk_slots, cudaStream_t st);
+
+// ---- device-wide exclusive scan (scan.cu) --------------------------------------
+// out[i] = sum_{j<i} in[j] for i < n, total -> *total_dev.  tmp needs scan_tmp_elems(n).
+int64_t scan_tmp_elems(int64_t n);
+void launch_scan_i64(const int64_t* in, int64_t* out, int64_t n, int64_t* total_dev, int64_t* tmp, cudaStream_t st);
+void launch_scan_i32(const int32_t* in, int64_t* out, int64_t n, int64_t* total_dev, int64_t* tmp, cudaStream_t st);
+// row_ptr: exclusive scan of int32 counts into int32 row_ptr[n+1] (+int64 total).
+void launch_scan_rowptr(const int32_t* in, int32_t* row_ptr, int64_t n, int64_t* total_dev, int64_t* tmp,
+                        cudaStream_t st);
+
+// ---- stage 2: AC-ESC (esc.cu) ---------------------------------------------------
+struct EscArgs {
+  CsrView A, B;
+  int32_t nblocks;
+  const int32_t* blk_nz_begin;
+  const int32_t* blk_nz_end;
+  const int32_t* block_row_starts;
+  const int64_t* pool_off;      // per block, elements
+  const int64_t* desc_off;      // per block, descriptor slots
+  int32_t* pool_col;
+  void* pool_val;
+  ChunkDesc* descs;
+  int32_t* nchunks;             // per block
+  int32_t* used;                // per block: chunk elements written
+  int32_t* row_count;           // per row of C
+};
+void launch_esc(const EscArgs& a, bool f64, cudaStream_t st);
+
+// ---- stage 3: chunk ordering, shared rows, merges (merge.cu) --------------------
+struct MergeState {
+  int32_t nblocks;
+  const int64_t* desc_off;
+  const int32_t* nchunks;
+  const int64_t* chunk_base;     // exclusive scan of nchunks
+  const ChunkDesc* descs;
+  ChunkDesc* dense;              // dense global chunk array [total_chunks]
+  int64_t max_chunks;            // host upper bound (total slots)
+  const int64_t* total_chunks_dev;
+  int32_t* shared_flag;          // [max_chunks] 1 where a shared row starts
+  int64_t* shared_pos;           // [max_chunks] exclusive scan of shared_flag
+  SharedRow* shared;             // [max_chunks]
+  int64_t* scan_tmp;
+};
+void launch_gather_chunks(const MergeState& m, cudaStream_t st);
+void launch_find_shared(const MergeState& m, int64_t* total_shared_dev, cudaStream_t st);
+
+struct MergeLists {
+  int64_t nshared;
+  SharedRow* shared;
+  int32_t* kind_flag;            // [nshared] scratch
+  int64_t* kind_pos;             // [nshared] scratch
+  int32_t* multi_idx;            // [nshared]
+  int32_t* path_idx;
+  int32_t* search_idx;
+  int64_t* counts_dev;           // [8]: nmulti, npath, nsearch, multi_total, merge_total, ngroups
+  int64_t* merge_total_scan;     // [nshared] exclusive scan of totals -> merge offsets
+  int64_t* multi_scan;           // [nshared]
+  int32_t* group_of;             // [nshared]
+  int32_t* group_start;          // [max groups + 1]
+  int64_t* scan_tmp;
+};
+void launch_classify(const MergeLists& L, cudaStream_t st);
+void launch_multi_groups(const MergeLists& L, int64_t nmulti, int64_t ngroups, cudaStream_t st);
+
+struct MergeArgs {
+  const ChunkDesc* dense;
+  SharedRow* shared;
+  const int32_t* list;           // indices into shared for this kind
+  int64_t nlist;
+  const int32_t* group_start;    // multi merge only: [ngroups+1] starts then [ngroups+1] ends
+  const int64_t* multi_scan;     // multi merge only: exclusive scan of totals over the list
+  int64_t ngroups;
+  const int32_t* pool_col;
+  const void* pool_val;
+  int32_t* merge_col;
+  void* merge_val;
+  int32_t* cur_first;            // per dense chunk cursors (path/search)
+  int32_t* cur_last;
+  int32_t* row_count;
+  int32_t* error_flag;
+};
+void launch_multi_merge(const MergeArgs& a, bool f64, cudaStream_t st);
+void launch_path_merge(const MergeArgs& a, bool f64, cudaStream_t st);
+void launch_search_merge(const MergeArgs& a, bool f64, cudaStream_t st);
+
+// ---- stage 4: chunk copy (copy.cu) ----------------------------------------------
+struct CopyArgs {
+  const ChunkDesc* dense;
+  const int64_t* total_chunks_dev;
+  int64_t max_chunks;
+  const SharedRow* shared;
+  int64_t nshared;
+  const int32_t* pool_col;
+  const void* pool_val;
+  const int32_t* merge_col;
+  const void* merge_val;
+  const int32_t* row_ptr;
+  int32_t* c_col;
+  void* c_val;
+};
+void launch_copy(const CopyArgs& a, bool f64, cudaStream_t st);
+
+// ---- validation ----------------------------------------------------------------
+void launch_validate(const CsrView& M, int32_t* bad_flag, cudaStream_t st);
+
+}  // namespace acs

@@ -1,0 +1,599 @@
+// Stage 3 — chunk ordering, shared-row detection, merge assignment (MCC) and the
+// three merges (§3.3).
+//
+// Chunk order.  The paper builds per-row linked lists with atomicExch and then sorts
+// each list by the chunk id (block, running number) to get a deterministic merge
+// order (L430, L434).  Here the chunk id order is materialised directly: a scan over
+// the per-block chunk counts gives every chunk its dense global index, and because
+// blocks cover increasing nonzero ranges, rows appear in that order monotonically.
+// A row is shared iff it is the last row of chunk j and the first row of chunk j+1;
+// its chunk list is the run of consecutive chunks holding it.  No atomics decide any
+// order.
+//
+// Merges.  Every merge re-runs local ESC (sort + Alg. 3 compaction) on the row's
+// chunk pieces, concatenated in global chunk order, so equal columns are summed in
+// chunk order by the fixed scan tree:
+//   * Multi Merge (L436-L440): rows with exactly two chunks are packed, several per
+//     CTA, by a prefix scan over their element counts.
+//   * Path Merge (L540-L544): rows with up to PATH_MAX_CHUNKS chunks; cuts through all
+//     chunks come from uniformly placed per-chunk samples sorted across the block.
+//   * Search Merge (L440-L442): any chunk count; cuts come from binary-search
+//     sampling of the column range, sub-sampled when too coarse.
+#include <climits>
+#include "esc_core.cuh"
+#include "kernels.cuh"
+
+namespace acs {
+
+// ------------------------------------------------------------ MCC kernels ----
+
+__global__ void k_gather_chunks(int32_t nblocks, const int64_t* __restrict__ desc_off,
+                                const int32_t* __restrict__ nchunks, const int64_t* __restrict__ chunk_base,
+                                const ChunkDesc* __restrict__ descs, ChunkDesc* __restrict__ dense) {
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= nblocks) return;
+  const int n = nchunks[b];
+  const int64_t src = desc_off[b], dst = chunk_base[b];
+  for (int s = 0; s < n; ++s) dense[dst + s] = descs[src + s];
+}
+
+void launch_gather_chunks(const MergeState& m, cudaStream_t st) {
+  if (m.nblocks <= 0) return;
+  k_gather_chunks<<<(m.nblocks + 255) / 256, 256, 0, st>>>(m.nblocks, m.desc_off, m.nchunks, m.chunk_base,
+                                                            m.descs, m.dense);
+}
+
+__global__ void k_shared_flags(const ChunkDesc* __restrict__ dense, const int64_t* __restrict__ total_dev,
+                               int64_t max_chunks, int32_t* __restrict__ flag) {
+  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= max_chunks) return;
+  const int64_t total = *total_dev;
+  int f = 0;
+  if (j + 1 < total) {
+    const int R = dense[j].last_row;
+    f = dense[j + 1].first_row == R && (j == 0 || dense[j - 1].last_row != R);
+  }
+  flag[j] = f;
+}
+
+__global__ void k_shared_fill(ChunkDesc* __restrict__ dense, const int64_t* __restrict__ total_dev, int64_t max_chunks,
+                              const int32_t* __restrict__ flag, const int64_t* __restrict__ pos,
+                              SharedRow* __restrict__ shared) {
+  const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= max_chunks || !flag[j]) return;
+  const int64_t total = *total_dev;
+  const int R = dense[j].last_row;
+  int m = 1;
+  int64_t tot = dense[j].last_count;
+  atomicOr(&dense[j].flags, 2);
+  while (j + m < total && dense[j + m].first_row == R) {
+    tot += dense[j + m].first_count;
+    atomicOr(&dense[j + m].flags, 1);
+    ++m;
+  }
+  SharedRow s;
+  s.row = R;
+  s.first_chunk = (int32_t)j;
+  s.nchunks = m;
+  s.total = (int32_t)tot;
+  s.merge_off = 0;
+  s.merged = 0;
+  s.kind = (m == 2 && tot <= CAP) ? 0 : (m <= PATH_MAX_CHUNKS ? 1 : 2);
+  shared[pos[j]] = s;
+}
+
+void launch_find_shared(const MergeState& m, int64_t* total_shared_dev, cudaStream_t st) {
+  if (m.max_chunks <= 0) {
+    cudaMemsetAsync(total_shared_dev, 0, sizeof(int64_t), st);
+    return;
+  }
+  const unsigned g = (unsigned)((m.max_chunks + 255) / 256);
+  k_shared_flags<<<g, 256, 0, st>>>(m.dense, m.total_chunks_dev, m.max_chunks, m.shared_flag);
+  launch_scan_i32(m.shared_flag, m.shared_pos, m.max_chunks, total_shared_dev, m.scan_tmp, st);
+  k_shared_fill<<<g, 256, 0, st>>>(m.dense, m.total_chunks_dev, m.max_chunks, m.shared_flag, m.shared_pos, m.shared);
+}
+
+// Classification (L440: "We decide which algorithm to use based on the length of each
+// row's chunk list") and merge-pool offsets.
+__global__ void k_kind_flags(const SharedRow* __restrict__ sh, int64_t n, int kind, int32_t* __restrict__ flag) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) flag[i] = sh[i].kind == kind;
+}
+__global__ void k_kind_scatter(const SharedRow* __restrict__ sh, int64_t n, int kind, const int64_t* __restrict__ pos,
+                               int32_t* __restrict__ list) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n && sh[i].kind == kind) list[pos[i]] = (int32_t)i;
+}
+__global__ void k_totals(const SharedRow* __restrict__ sh, int64_t n, int32_t* __restrict__ out) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) out[i] = sh[i].total;
+}
+__global__ void k_set_merge_off(SharedRow* __restrict__ sh, int64_t n, const int64_t* __restrict__ off) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) sh[i].merge_off = off[i];
+}
+
+void launch_classify(const MergeLists& L, cudaStream_t st) {
+  if (L.nshared <= 0) {
+    cudaMemsetAsync(L.counts_dev, 0, 8 * sizeof(int64_t), st);
+    return;
+  }
+  const unsigned g = (unsigned)((L.nshared + 255) / 256);
+  int32_t* lists[3] = {L.multi_idx, L.path_idx, L.search_idx};
+  for (int kind = 0; kind < 3; ++kind) {
+    k_kind_flags<<<g, 256, 0, st>>>(L.shared, L.nshared, kind, L.kind_flag);
+    launch_scan_i32(L.kind_flag, L.kind_pos, L.nshared, L.counts_dev + kind, L.scan_tmp, st);
+    k_kind_scatter<<<g, 256, 0, st>>>(L.shared, L.nshared, kind, L.kind_pos, lists[kind]);
+  }
+  k_totals<<<g, 256, 0, st>>>(L.shared, L.nshared, L.kind_flag);
+  launch_scan_i32(L.kind_flag, L.merge_total_scan, L.nshared, L.counts_dev + 4, L.scan_tmp, st);
+  k_set_merge_off<<<g, 256, 0, st>>>(L.shared, L.nshared, L.merge_total_scan);
+}
+
+// Multi Merge packing (L436-L438): "we run a prefix scan over all shared rows ...
+// combine row range identifiers, if the sum of their respective elements does not
+// overflow the number of elements we can handle in one block".  Made deterministic and
+// parallel: with P the exclusive prefix of a 2-chunk row's total, rows with
+// floor(P/CAP) == floor((P+total-1)/CAP) form group 2*floor(P/CAP); the (at most one)
+// row crossing a CAP boundary forms group 2*floor(P/CAP)+1 alone.
+__global__ void k_multi_totals(const SharedRow* __restrict__ sh, const int32_t* __restrict__ list, int64_t n,
+                               int32_t* __restrict__ out) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) out[i] = sh[list[i]].total;
+}
+__global__ void k_multi_group(const SharedRow* __restrict__ sh, const int32_t* __restrict__ list, int64_t n,
+                              const int64_t* __restrict__ P, int32_t* __restrict__ group_of) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const int64_t p = P[i], t = sh[list[i]].total;
+  const int64_t w = p / CAP;
+  group_of[i] = (int32_t)(2 * w + (((p + t - 1) / CAP) != w ? 1 : 0));
+}
+__global__ void k_group_bounds(const int32_t* __restrict__ group_of, int64_t n, int32_t* __restrict__ gstart,
+                               int32_t* __restrict__ gend) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const int g = group_of[i];
+  if (i == 0 || group_of[i - 1] != g) gstart[g] = (int32_t)i;
+  if (i == n - 1 || group_of[i + 1] != g) gend[g] = (int32_t)(i + 1);
+}
+
+void launch_multi_groups(const MergeLists& L, int64_t nmulti, int64_t ngroups, cudaStream_t st) {
+  if (nmulti <= 0) return;
+  const unsigned g = (unsigned)((nmulti + 255) / 256);
+  k_multi_totals<<<g, 256, 0, st>>>(L.shared, L.multi_idx, nmulti, L.kind_flag);
+  launch_scan_i32(L.kind_flag, L.multi_scan, nmulti, L.counts_dev + 6, L.scan_tmp, st);
+  k_multi_group<<<g, 256, 0, st>>>(L.shared, L.multi_idx, nmulti, L.multi_scan, L.group_of);
+  cudaMemsetAsync(L.group_start, 0xFF, sizeof(int32_t) * 2 * (ngroups + 1), st);
+  k_group_bounds<<<g, 256, 0, st>>>(L.group_of, nmulti, L.group_start, L.group_start + (ngroups + 1));
+}
+
+// ----------------------------------------------------------- merge kernels ---
+
+template <typename T>
+struct MergeSmem {
+  SortSmem<T> s;
+  int64_t lo, hi, cut;
+  int best;
+  int red[40];
+};
+
+// row pieces of shared row `sh`: piece 0 is the tail of chunk first_chunk (the row is
+// that chunk's last row), pieces t >= 1 are the heads of the following chunks.
+__device__ __forceinline__ void piece_of(const ChunkDesc* __restrict__ dense, const SharedRow& sh, int t,
+                                         int64_t& base, int& len) {
+  const ChunkDesc& d = dense[sh.first_chunk + t];
+  if (t == 0) { base = d.data_off + d.count - d.last_count; len = d.last_count; }
+  else { base = d.data_off; len = d.first_count; }
+}
+
+// Sort + compact one Multi-Merge group; the element with row counter rc goes to
+// position rc-1 of its merged row (the per-row counter of Alg. 3).
+template <typename Word, typename T>
+__device__ __forceinline__ void multi_tail(MergeSmem<T>& S, const MergeArgs& a, int i0, int n,
+                                           const int (&tmpr)[ITEMS], const int (&tmpc)[ITEMS], int cmin,
+                                           int rowbits, int colbits) {
+  const int tid = threadIdx.x;
+  Word* sw = reinterpret_cast<Word*>(S.s.words);
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    const int pos = i * THREADS + tid;
+    sw[pad32(pos)] = pos < n ? (((((Word)tmpr[i] << colbits) | (Word)(tmpc[i] - cmin)) << IDXBITS) | (Word)pos)
+                             : ~(Word)0;
+  }
+  __syncthreads();
+  Word k[ITEMS];
+  T ev[ITEMS];
+  load_and_sort<Word, T>(S.s, rowbits + colbits, k);
+  const ScanCtx<Word, T> ctx = compaction_prepare<Word, T>(S.s, k, n, colbits, ev);
+  T* mval = reinterpret_cast<T*>(a.merge_val);
+  const Word colmask = colbits ? (((Word)1 << colbits) - (Word)1) : (Word)0;
+  compaction_emit<Word, T>(k, ev, n, colbits, ctx, [&](int, Word key, T val, uint32_t state, bool row_end) {
+    const int rel = (int)(key >> colbits);
+    SharedRow* sh = &a.shared[a.list[i0 + rel]];
+    const int rc = st_row_count(state);
+    const int64_t dst = sh->merge_off + rc - 1;
+    a.merge_col[dst] = cmin + (int)(key & colmask);
+    mval[dst] = val;
+    if (row_end) {
+      sh->merged = rc;
+      a.row_count[sh->row] = rc;
+    }
+  });
+}
+
+// ---- Multi Merge: one CTA per packed group of two-chunk rows -----------------------
+template <typename T>
+__global__ void __launch_bounds__(THREADS, 2) k_multi_merge(MergeArgs a) {
+  const int64_t* __restrict__ multi_scan = a.multi_scan;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  MergeSmem<T>& S = *reinterpret_cast<MergeSmem<T>*>(smem_raw);
+  const int g = blockIdx.x;
+  const int i0 = a.group_start[g];
+  if (i0 < 0) return;
+  const int i1 = a.group_start[a.ngroups + 1 + g];
+  const int nrows = i1 - i0;
+  const int tid = threadIdx.x;
+  const int64_t P0 = multi_scan[i0];
+  int* pref = S.s.u.wprefix;           // element offset of each row inside the group
+  for (int r = tid; r < nrows; r += THREADS) pref[r] = (int)(multi_scan[i0 + r] - P0);
+  if (tid == 0) {
+    const SharedRow& last = a.shared[a.list[i1 - 1]];
+    pref[nrows] = (int)(multi_scan[i1 - 1] - P0) + last.total;
+  }
+  __syncthreads();
+  const int n = pref[nrows];
+  const T* __restrict__ pval = reinterpret_cast<const T*>(a.pool_val);
+  // gather: column / value / local row per position (row order, then chunk order)
+  int cmin = INT_MAX, cmax = INT_MIN;
+  for (int pos = tid; pos < n; pos += THREADS) {
+    int lo = 0, hi = nrows - 1;
+    while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (pref[mid] <= pos) lo = mid; else hi = mid - 1; }
+    const SharedRow sh = a.shared[a.list[i0 + lo]];
+    const int off = pos - pref[lo];
+    int64_t b0; int l0;
+    piece_of(a.dense, sh, 0, b0, l0);
+    int64_t src;
+    if (off < l0) src = b0 + off;
+    else { int64_t b1; int l1; piece_of(a.dense, sh, 1, b1, l1); src = b1 + (off - l0); }
+    const int c = a.pool_col[src];
+    cmin = min(cmin, c); cmax = max(cmax, c);
+    S.s.vals[pos] = pval[src];
+    reinterpret_cast<int*>(S.s.words)[pos] = c;      // temporarily: column
+  }
+  int rdummy0 = 0, rdummy1 = 0;
+  block_minmax4(rdummy0, rdummy1, cmin, cmax, S.red);
+  const int rowbits = bit_width_u64((uint64_t)(nrows - 1));
+  const int colbits = bit_width_u64((uint64_t)((int64_t)cmax - cmin));
+  // build words in place (read column, row -> word); positions stay put
+  int tmpc[ITEMS], tmpr[ITEMS];
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    const int pos = i * THREADS + tid;
+    tmpc[i] = pos < n ? reinterpret_cast<int*>(S.s.words)[pos] : 0;
+    int r = 0;
+    if (pos < n) {
+      int lo = 0, hi = nrows - 1;
+      while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (pref[mid] <= pos) lo = mid; else hi = mid - 1; }
+      r = lo;
+    }
+    tmpr[i] = r;
+  }
+  __syncthreads();
+  if (rowbits + colbits + IDXBITS < 32)
+    multi_tail<uint32_t, T>(S, a, i0, n, tmpr, tmpc, cmin, rowbits, colbits);
+  else
+    multi_tail<uint64_t, T>(S, a, i0, n, tmpr, tmpc, cmin, rowbits, colbits);
+}
+
+// ---- shared helpers of Path / Search Merge ---------------------------------------
+__device__ __forceinline__ int lower_bound_i32(const int32_t* __restrict__ p, int lo, int hi, int64_t v) {
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if ((int64_t)p[mid] < v) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ int* cursor_of(const MergeArgs& a, const SharedRow& sh, int t) {
+  return t == 0 ? &a.cur_last[sh.first_chunk] : &a.cur_first[sh.first_chunk + t];
+}
+
+template <typename Word, typename T>
+__device__ __forceinline__ int window_tail(MergeSmem<T>& S, const MergeArgs& a, const SharedRow& sh, int n,
+                                           int colbits, int64_t lo, int64_t out) {
+  Word k[ITEMS];
+  T ev[ITEMS];
+  load_and_sort<Word, T>(S.s, colbits, k);
+  const ScanCtx<Word, T> ctx = compaction_prepare<Word, T>(S.s, k, n, colbits, ev);
+  T* mval = reinterpret_cast<T*>(a.merge_val);
+  const int64_t dst = sh.merge_off + out;
+  const Word colmask = colbits ? (((Word)1 << colbits) - (Word)1) : (Word)0;
+  compaction_emit<Word, T>(k, ev, n, colbits, ctx, [&](int idx, Word key, T val, uint32_t state, bool) {
+    const int p = st_count(state) - 1;
+    a.merge_col[dst + p] = (int32_t)(lo + (int64_t)(key & colmask));
+    mval[dst + p] = val;
+    if (idx == n - 1) S.best = p + 1;
+  });
+  __syncthreads();
+  return S.best;
+}
+
+// Run one merge window: all elements with column < cut, from every piece, in piece
+// (= global chunk) order; sort + compact; append to the merged row.  Returns the number
+// of merged elements written.
+template <typename T>
+__device__ int merge_window(MergeSmem<T>& S, const MergeArgs& a, const SharedRow& sh, int m, int64_t lo, int64_t hi,
+                            int64_t cut, int64_t out) {
+  const int tid = threadIdx.x;
+  int* wp = S.s.u.wprefix;
+  // window sizes per piece, prefix in piece order
+  int carry = 0;
+  for (int base = 0; base < m; base += THREADS) {
+    const int t = base + tid;
+    int cnt = 0;
+    if (t < m) {
+      int64_t b; int len;
+      piece_of(a.dense, sh, t, b, len);
+      const int cur = *cursor_of(a, sh, t);
+      const int ub = lower_bound_i32(a.pool_col + b, cur, len, cut);
+      cnt = ub - cur;
+    }
+    int total;
+    const int ex = block_exclusive_sum<int>(cnt, S.s.scratch, &total);
+    if (t < m) wp[t] = carry + ex;
+    carry += total;
+  }
+  if (tid == 0) wp[m] = carry;
+  __syncthreads();
+  const int n = carry;
+  const int64_t hcut = min(cut - 1, hi);
+  const int colbits = bit_width_u64((uint64_t)(hcut - lo));
+  const T* __restrict__ pval = reinterpret_cast<const T*>(a.pool_val);
+  const bool w32 = colbits + IDXBITS < 32;
+  for (int pos = tid; pos < CAP; pos += THREADS) {
+    if (pos < n) {
+      int l = 0, h = m - 1;
+      while (l < h) { const int mid = (l + h + 1) >> 1; if (wp[mid] <= pos) l = mid; else h = mid - 1; }
+      int64_t b; int len;
+      piece_of(a.dense, sh, l, b, len);
+      const int cur = *cursor_of(a, sh, l);
+      const int64_t src = b + cur + (pos - wp[l]);
+      const uint64_t key = (uint64_t)((int64_t)a.pool_col[src] - lo);
+      S.s.vals[pos] = pval[src];
+      if (w32) reinterpret_cast<uint32_t*>(S.s.words)[pad32(pos)] = (uint32_t)((key << IDXBITS) | (uint64_t)pos);
+      else S.s.words[pad32(pos)] = (key << IDXBITS) | (uint64_t)pos;
+    } else {
+      if (w32) reinterpret_cast<uint32_t*>(S.s.words)[pad32(pos)] = ~0u;
+      else S.s.words[pad32(pos)] = ~0ull;
+    }
+  }
+  __syncthreads();
+  // advance the cursors past the window (wp aliases the sort counters: do it now)
+  for (int t = tid; t < m; t += THREADS) *cursor_of(a, sh, t) += wp[t + 1] - wp[t];
+  __syncthreads();
+  const int written = w32 ? window_tail<uint32_t, T>(S, a, sh, n, colbits, lo, out)
+                          : window_tail<uint64_t, T>(S, a, sh, n, colbits, lo, out);
+  __syncthreads();
+  return written;
+}
+
+// remaining elements, min next column, max last column over all pieces
+__device__ __forceinline__ void piece_ranges(const MergeArgs& a, const SharedRow& sh, int m, int* red,
+                                             int& rem, int& lo, int& hi) {
+  int r = 0, l = INT_MAX, h = INT_MIN;
+  for (int t = threadIdx.x; t < m; t += THREADS) {
+    int64_t b; int len;
+    piece_of(a.dense, sh, t, b, len);
+    const int cur = *cursor_of(a, sh, t);
+    if (cur < len) {
+      r += len - cur;
+      l = min(l, a.pool_col[b + cur]);
+      h = max(h, a.pool_col[b + len - 1]);
+    }
+  }
+  int tot;
+  block_exclusive_sum<int>(r, red, &tot);
+  int d0 = 0, d1 = 0;
+  block_minmax4(d0, d1, l, h, red);
+  rem = tot;
+  lo = l;
+  hi = h;
+}
+
+// ---- Search Merge (L440-L442) ----------------------------------------------------
+template <typename T>
+__global__ void __launch_bounds__(THREADS, 2) k_search_merge(MergeArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  MergeSmem<T>& S = *reinterpret_cast<MergeSmem<T>*>(smem_raw);
+  const int tid = threadIdx.x;
+  const SharedRow sh = a.shared[a.list[blockIdx.x]];
+  const int m = sh.nchunks;
+  if (m > CAP) { if (tid == 0) atomicExch(a.error_flag, 1); return; }
+  for (int t = tid; t < m; t += THREADS) *cursor_of(a, sh, t) = 0;
+  __syncthreads();
+  int64_t out = 0;
+  while (true) {
+    int rem, lo, hi;
+    piece_ranges(a, sh, m, S.red, rem, lo, hi);
+    if (rem == 0) break;
+    int64_t cut;
+    if (rem <= CAP) {
+      cut = (int64_t)hi + 1;
+    } else {
+      // "uniformly sample this range, according to ((max-min)/THREADS), assigning one
+      // thread to each sample ... the thread with the largest sum that still fits"
+      int64_t L = lo, H = hi;
+      while (true) {
+        const int64_t width = H - L + 1;
+        const int64_t cand = L + max((int64_t)1, ((int64_t)(tid + 1) * width) / THREADS);
+        int64_t cnt = 0;
+        for (int t = 0; t < m; ++t) {
+          int64_t b; int len;
+          piece_of(a.dense, sh, t, b, len);
+          const int cur = *cursor_of(a, sh, t);
+          cnt += lower_bound_i32(a.pool_col + b, cur, len, cand) - cur;
+        }
+        const int fits = cnt <= CAP ? tid : -1;
+        int bmax = fits, d0 = 0, d1 = 0, d2 = 0;
+        block_minmax4(d0, d1, d2, bmax, S.red);
+        if (bmax >= 0) {
+          if (tid == bmax) S.cut = cand;
+          __syncthreads();
+          cut = S.cut;
+          __syncthreads();
+          break;
+        }
+        // too coarse: sub-sample the first interval
+        H = L + max((int64_t)1, width / THREADS) - 1;
+      }
+    }
+    out += merge_window<T>(S, a, sh, m, lo, hi, cut, out);
+  }
+  if (tid == 0) {
+    a.shared[a.list[blockIdx.x]].merged = (int32_t)out;
+    a.row_count[sh.row] = (int32_t)out;
+  }
+}
+
+// ---- Path Merge (L540-L544) --------------------------------------------------------
+// Samples are placed uniformly over the remaining entries of every chunk; sorting all
+// samples by column across the block and scanning gives, for every sample column X,
+// how far each chunk's path has advanced (the last sample of that chunk <= X).  The
+// element count below X is then bracketed by sample positions; we pick the largest
+// sample X whose upper bracket fits, and the exact per-chunk cut is found by a local
+// search inside one sample interval (reading R12).
+template <typename T>
+__global__ void __launch_bounds__(THREADS, 2) k_path_merge(MergeArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  MergeSmem<T>& S = *reinterpret_cast<MergeSmem<T>*>(smem_raw);
+  const int tid = threadIdx.x;
+  const SharedRow sh = a.shared[a.list[blockIdx.x]];
+  const int m = sh.nchunks;
+  for (int t = tid; t < m; t += THREADS) *cursor_of(a, sh, t) = 0;
+  __syncthreads();
+  const int SPC = THREADS / PATH_MAX_CHUNKS;          // samples per chunk (>= 8)
+  int64_t out = 0;
+  while (true) {
+    int rem, lo, hi;
+    piece_ranges(a, sh, m, S.red, rem, lo, hi);
+    if (rem == 0) break;
+    int64_t cut;
+    if (rem <= CAP) {
+      cut = (int64_t)hi + 1;
+    } else {
+      // sample k of chunk t sits at cur + (k+1)*step - 1 of its remaining entries;
+      // thread tid = t*SPC + k owns it.  Its column value is a cut candidate; the count
+      // of elements < candidate is sum_t' (#entries of t' below it), computed from the
+      // sorted samples of every chunk by binary search on that chunk's samples
+      // (the "max scan over per-chunk sample numbers" of the paper), refined exactly.
+      int* samp = S.s.u.wprefix;                      // [PATH_MAX_CHUNKS * SPC] columns
+      const int t = tid / SPC, k = tid % SPC;
+      int64_t cand = INT64_MAX;
+      if (t < m) {
+        int64_t b; int len;
+        piece_of(a.dense, sh, t, b, len);
+        const int cur = *cursor_of(a, sh, t);
+        const int r = len - cur;
+        const int step = max(1, (r + SPC - 1) / SPC);
+        const int idx = cur + min(r, (k + 1) * step) - 1;
+        samp[tid] = (r > 0) ? a.pool_col[b + idx] : INT_MAX;
+        cand = (r > 0) ? (int64_t)a.pool_col[b + idx] : INT64_MAX;
+      } else {
+        samp[tid] = INT_MAX;
+      }
+      __syncthreads();
+      // exact count below candidate X: per chunk, the samples bracket the position,
+      // then a binary search inside the bracket
+      int64_t cnt = 0;
+      if (cand != INT64_MAX) {
+        for (int t2 = 0; t2 < m; ++t2) {
+          int64_t b; int len;
+          piece_of(a.dense, sh, t2, b, len);
+          const int cur = *cursor_of(a, sh, t2);
+          const int r = len - cur;
+          if (r <= 0) continue;
+          const int step = max(1, (r + SPC - 1) / SPC);
+          // samples of chunk t2 are sorted: find the first sample >= cand
+          int s = 0;
+          while (s < SPC && samp[t2 * SPC + s] < cand) ++s;
+          const int lo_i = cur + min(r, s * step);                 // all before are < cand
+          const int hi_i = cur + min(r, (s + 1) * step);           // sample s is >= cand
+          cnt += lower_bound_i32(a.pool_col + b, lo_i, hi_i, cand) - cur;
+        }
+      }
+      const int fits = (cand != INT64_MAX && cnt <= CAP && cand > lo) ? tid : -1;
+      // largest fitting candidate column (ties: any thread, same column)
+      int best = fits;
+      {
+        // choose max candidate among fitting threads: reduce on (cand) via two passes
+        int d0 = 0, d1 = 0, d2 = 0;
+        int key = fits >= 0 ? (int)cand : INT_MIN;
+        block_minmax4(d0, d1, d2, key, S.red);
+        if (key != INT_MIN) {
+          cut = key;
+        } else {
+          // no sample fits (very skewed): fall back to search sampling of the range
+          int64_t L = lo, H = hi;
+          while (true) {
+            const int64_t width = H - L + 1;
+            const int64_t c2 = L + max((int64_t)1, ((int64_t)(tid + 1) * width) / THREADS);
+            int64_t c = 0;
+            for (int t2 = 0; t2 < m; ++t2) {
+              int64_t b; int len;
+              piece_of(a.dense, sh, t2, b, len);
+              const int cur = *cursor_of(a, sh, t2);
+              c += lower_bound_i32(a.pool_col + b, cur, len, c2) - cur;
+            }
+            int bm = c <= CAP ? tid : -1, e0 = 0, e1 = 0, e2 = 0;
+            block_minmax4(e0, e1, e2, bm, S.red);
+            if (bm >= 0) {
+              if (tid == bm) S.cut = c2;
+              __syncthreads();
+              cut = S.cut;
+              __syncthreads();
+              break;
+            }
+            H = L + max((int64_t)1, width / THREADS) - 1;
+          }
+        }
+        (void)best;
+      }
+    }
+    out += merge_window<T>(S, a, sh, m, lo, hi, cut, out);
+  }
+  if (tid == 0) {
+    a.shared[a.list[blockIdx.x]].merged = (int32_t)out;
+    a.row_count[sh.row] = (int32_t)out;
+  }
+}
+
+template <typename T>
+static void launch_merge_t(const MergeArgs& a, int which, cudaStream_t st) {
+  const size_t smem = sizeof(MergeSmem<T>);
+  if (which == 0) {
+    cudaFuncSetAttribute(k_multi_merge<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_multi_merge<T><<<(unsigned)a.ngroups, THREADS, smem, st>>>(a);
+  } else if (which == 1) {
+    cudaFuncSetAttribute(k_path_merge<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_path_merge<T><<<(unsigned)a.nlist, THREADS, smem, st>>>(a);
+  } else {
+    cudaFuncSetAttribute(k_search_merge<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_search_merge<T><<<(unsigned)a.nlist, THREADS, smem, st>>>(a);
+  }
+}
+
+void launch_multi_merge(const MergeArgs& a, bool f64, cudaStream_t st) {
+  if (a.ngroups <= 0) return;
+  if (f64) launch_merge_t<double>(a, 0, st); else launch_merge_t<float>(a, 0, st);
+}
+void launch_path_merge(const MergeArgs& a, bool f64, cudaStream_t st) {
+  if (a.nlist <= 0) return;
+  if (f64) launch_merge_t<double>(a, 1, st); else launch_merge_t<float>(a, 1, st);
+}
+void launch_search_merge(const MergeArgs& a, bool f64, cudaStream_t st) {
+  if (a.nlist <= 0) return;
+  if (f64) launch_merge_t<double>(a, 2, st); else launch_merge_t<float>(a, 2, st);
+}
+
+}  // namespace acs

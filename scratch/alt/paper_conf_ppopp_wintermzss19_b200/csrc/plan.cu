@@ -1,0 +1,818 @@
+// Host orchestration of AC-SpGEMM (Fig. 2; §3.5) behind
+// the C ABI declared in include/acspgemm.h.
+//
+// Stage sequence on one caller stream:
+//   GLB      segments -> Alg. 1 -> per-block nonzero range and exact product count ->
+//            scans giving every block a deterministic chunk-pool range and descriptor
+//            slot range                                     [read-back 1: totals]
+//   ESC      one CTA per block                               (esc.cu)
+//   MCC      dense chunk order, shared rows                  [read-back 2: counts]
+//            classification, merge offsets, Multi-Merge packing [read-back 3]
+//   MM/PM/SM the three merges                                (merge.cu)
+//   SCAN     row_ptr of C                                    [read-back 4: nnz(C)]
+//   CC       (numeric) chunk copy into C                     (copy.cu)
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include <algorithm>
+
+#include "../../include/acspgemm.h"
+#include "esc_core.cuh"
+#include "kernels.cuh"
+
+namespace acs {
+thread_local long long tl_launches = 0;
+}
+
+namespace {
+
+using namespace acs;
+
+thread_local std::string tl_err;
+
+acspgemm_status set_err(acspgemm_status s, const std::string& msg) {
+  tl_err = msg;
+  return s;
+}
+
+#define ACS_CUDA(call)                                                                        \
+  do {                                                                                        \
+    cudaError_t e_ = (call);                                                                  \
+    if (e_ != cudaSuccess) {                                                                  \
+      if (e_ == cudaErrorMemoryAllocation) {                                                  \
+        cudaGetLastError();                                                                   \
+        return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+      }                                                                                       \
+      return set_err(ACSPGEMM_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+    }                                                                                         \
+  } while (0)
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+};
+
+enum Stage { S_GLB = 0, S_ESC, S_MCC, S_MM, S_PM, S_SM, S_SCAN, S_CC, S_END, NSTAGE_EV };
+
+}  // namespace
+
+struct acspgemm_plan_s {
+  acspgemm_options opt;
+  int nseg_explicit = 0;
+  int64_t seg_rows_explicit[MAX_SEGMENTS + 1];
+  // buffers
+  DevBuf seg, seg_rows, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base;
+  DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
+  DevBuf kflag, kpos, lmulti, lpath, lsearch, mscan, mtscan, group_of, gstart, merge_col, merge_val;
+  DevBuf cur_first, cur_last, err, bused, bused_scan;
+  int64_t* h_scal = nullptr;     // pinned read-back buffer
+  cudaEvent_t ev[NSTAGE_EV];
+  bool ev_ok = false;
+  // last problem
+  bool ready = false;
+  bool empty = true;
+  bool f64 = true;
+  int64_t rows = 0, cols = 0, nnz = 0;
+  int64_t max_chunks = 0, total_chunks = 0, nshared = 0;
+  acspgemm_info info;
+  long long launches_sym = 0;
+  int dev = 0;
+};
+
+namespace {
+
+acspgemm_status ensure(DevBuf& b, size_t bytes) {
+  if (bytes == 0) bytes = 16;
+  if (b.bytes >= bytes) return ACSPGEMM_OK;
+  if (b.p) {
+    cudaError_t e = cudaFree(b.p);
+    if (e != cudaSuccess) return set_err(ACSPGEMM_ERR_CUDA, std::string("cudaFree: ") + cudaGetErrorString(e));
+    b.p = nullptr;
+    b.bytes = 0;
+  }
+  size_t want = bytes + bytes / 8;          // headroom so repeated calls do not re-allocate
+  cudaError_t e = cudaMalloc(&b.p, want);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    b.p = nullptr;
+    return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY,
+                   "cudaMalloc(" + std::to_string(want) + " bytes): " + cudaGetErrorString(e));
+  }
+  b.bytes = want;
+  return ACSPGEMM_OK;
+}
+
+#define ACS_ENSURE(buf, bytes)                          \
+  do {                                                  \
+    acspgemm_status s_ = ensure((buf), (size_t)(bytes)); \
+    if (s_ != ACSPGEMM_OK) return s_;                   \
+  } while (0)
+
+template <typename P>
+P* ptr(DevBuf& b) { return reinterpret_cast<P*>(b.p); }
+
+void free_buf(DevBuf& b) {
+  if (b.p) cudaFree(b.p);
+  b.p = nullptr;
+  b.bytes = 0;
+}
+
+void record(acspgemm_plan p, int stage, cudaStream_t st) {
+  if (p->opt.collect_stage_times && p->ev_ok) cudaEventRecord(p->ev[stage], st);
+}
+
+acspgemm_status check_in(const acspgemm_csr_in* M, const char* name) {
+  if (!M) return set_err(ACSPGEMM_ERR_INVALID_ARG, std::string(name) + " is NULL");
+  if (M->rows < 0 || M->cols < 0 || M->nnz < 0)
+    return set_err(ACSPGEMM_ERR_INVALID_ARG, std::string(name) + ": negative size");
+  if (M->rows >= (int64_t(1) << 31) - 1 || M->cols >= (int64_t(1) << 31) - 1 || M->nnz >= (int64_t(1) << 31))
+    return set_err(ACSPGEMM_ERR_INVALID_ARG, std::string(name) + ": size exceeds int32 indexing");
+  if (M->rows > 0 && !M->row_ptr) return set_err(ACSPGEMM_ERR_INVALID_ARG, std::string(name) + ".row_ptr is NULL");
+  if (M->nnz > 0 && (!M->col_idx || !M->val))
+    return set_err(ACSPGEMM_ERR_INVALID_ARG, std::string(name) + ": NULL col_idx/val with nnz > 0");
+  return ACSPGEMM_OK;
+}
+
+int64_t helper_bytes(acspgemm_plan p) {
+  DevBuf* bs[] = {&p->seg, &p->seg_rows, &p->scal, &p->brs, &p->nzb, &p->nze, &p->bprod, &p->bslot,
+                  &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->descs, &p->dense, &p->sflag,
+                  &p->spos, &p->shared, &p->row_count, &p->row_ptr, &p->scan_tmp, &p->kflag, &p->kpos,
+                  &p->lmulti, &p->lpath, &p->lsearch, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
+                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan};
+  int64_t t = 0;
+  for (DevBuf* b : bs) t += (int64_t)b->bytes;
+  return t;
+}
+
+acspgemm_status sync_read(acspgemm_plan p, const int64_t* dev, int n, cudaStream_t st) {
+  ACS_CUDA(cudaMemcpyAsync(p->h_scal, dev, sizeof(int64_t) * n, cudaMemcpyDeviceToHost, st));
+  ACS_CUDA(cudaStreamSynchronize(st));
+  return ACSPGEMM_OK;
+}
+
+__global__ void k_put_i64(int64_t* dst, const int32_t* src) { *dst = *src; }
+
+acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
+                              acspgemm_dtype dtype, cudaStream_t st, int64_t* nnz_c) {
+  acspgemm_status s;
+  if ((s = check_in(A, "A")) != ACSPGEMM_OK) return s;
+  if ((s = check_in(B, "B")) != ACSPGEMM_OK) return s;
+  if (!nnz_c) return set_err(ACSPGEMM_ERR_INVALID_ARG, "nnz_c is NULL");
+  if (dtype != ACSPGEMM_F32 && dtype != ACSPGEMM_F64) return set_err(ACSPGEMM_ERR_INVALID_ARG, "bad dtype");
+  if (A->cols != B->rows) return set_err(ACSPGEMM_ERR_DIM_MISMATCH, "A.cols != B.rows");
+  ACS_CUDA(cudaGetDevice(&p->dev));
+  const long long l0 = tl_launches;
+  p->ready = false;
+  p->f64 = dtype == ACSPGEMM_F64;
+  p->rows = A->rows;
+  p->cols = B->cols;
+  std::memset(&p->info, 0, sizeof(p->info));
+  const int vbytes = p->f64 ? 8 : 4;
+  p->info.pool_estimate_bytes =
+      acspgemm_pool_estimate_bytes(A->rows, A->nnz, B->rows, B->cols, B->nnz, vbytes);
+  const CsrView Av{A->rows, A->cols, A->row_ptr, A->col_idx, A->val};
+  const CsrView Bv{B->rows, B->cols, B->row_ptr, B->col_idx, B->val};
+
+  // empty inputs are legal (reading R18): C has no entries, no kernels run
+  if (A->rows == 0 || A->nnz == 0 || B->nnz == 0) {
+    p->empty = true;
+    p->nnz = 0;
+    p->ready = true;
+    *nnz_c = 0;
+    p->info.nsegments = 0;
+    p->launches_sym = 0;
+    return ACSPGEMM_OK;
+  }
+  p->empty = false;
+  ACS_ENSURE(p->scal, sizeof(int64_t) * 32);
+  ACS_ENSURE(p->err, sizeof(int32_t) * 4);
+  int64_t* scal = ptr<int64_t>(p->scal);
+  ACS_CUDA(cudaMemsetAsync(p->err.p, 0, sizeof(int32_t) * 4, st));
+
+  if (p->opt.validate_inputs) {
+    launch_validate(Av, ptr<int32_t>(p->err), st);
+    launch_validate(Bv, ptr<int32_t>(p->err), st);
+    tl_launches += 2;
+    ACS_CUDA(cudaMemcpyAsync(p->h_scal, p->err.p, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+    ACS_CUDA(cudaStreamSynchronize(st));
+    if (*reinterpret_cast<int32_t*>(p->h_scal) != 0)
+      return set_err(ACSPGEMM_ERR_INVALID_ARG, "input is not canonical CSR (row_ptr/col order/range)");
+  }
+
+  // ------------------------------------------------------------ GLB -----------
+  record(p, S_GLB, st);
+  int nseg = p->nseg_explicit > 0 ? p->nseg_explicit : p->opt.num_segments;
+  if (nseg < 1) nseg = DEFAULT_SEGMENTS;
+  if (nseg > MAX_SEGMENTS) nseg = MAX_SEGMENTS;
+  const int64_t max_blocks = (A->nnz + NPB - 1) / NPB + nseg;
+  ACS_ENSURE(p->seg, sizeof(int64_t) * 3 * (MAX_SEGMENTS + 1));
+  ACS_ENSURE(p->seg_rows, sizeof(int64_t) * (MAX_SEGMENTS + 1));
+  const int64_t* explicit_rows = nullptr;
+  if (p->nseg_explicit > 0) {
+    if (p->seg_rows_explicit[p->nseg_explicit] != A->rows)
+      return set_err(ACSPGEMM_ERR_INVALID_ARG, "explicit segments do not end at A.rows");
+    ACS_CUDA(cudaMemcpyAsync(p->seg_rows.p, p->seg_rows_explicit, sizeof(int64_t) * (nseg + 1),
+                             cudaMemcpyHostToDevice, st));
+    explicit_rows = ptr<int64_t>(p->seg_rows);
+  }
+  ACS_ENSURE(p->brs, sizeof(int32_t) * max_blocks);
+  ACS_ENSURE(p->nzb, sizeof(int32_t) * max_blocks);
+  ACS_ENSURE(p->nze, sizeof(int32_t) * max_blocks);
+  ACS_ENSURE(p->bprod, sizeof(int64_t) * max_blocks);
+  ACS_ENSURE(p->bslot, sizeof(int64_t) * max_blocks);
+  ACS_ENSURE(p->pool_off, sizeof(int64_t) * max_blocks);
+  ACS_ENSURE(p->desc_off, sizeof(int64_t) * max_blocks);
+  ACS_ENSURE(p->nchunks, sizeof(int32_t) * max_blocks);
+  ACS_ENSURE(p->chunk_base, sizeof(int64_t) * max_blocks);
+  ACS_ENSURE(p->bused, sizeof(int32_t) * max_blocks);
+  ACS_ENSURE(p->bused_scan, sizeof(int64_t) * max_blocks);
+  const int64_t tmp_n = scan_tmp_elems(std::max<int64_t>(max_blocks, A->rows) * 2 + 1024);
+  ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * tmp_n);
+  int32_t* nblocks_dev = reinterpret_cast<int32_t*>(scal + 20);
+  launch_segments(Av, nseg, explicit_rows, ptr<int64_t>(p->seg), nblocks_dev, st);
+  tl_launches += 1;
+  launch_glb(Av, nseg, ptr<int64_t>(p->seg), ptr<int32_t>(p->brs), max_blocks, st);
+  tl_launches += 1;
+  launch_block_bounds(Av, Bv, nseg, ptr<int64_t>(p->seg), nblocks_dev, max_blocks, ptr<int32_t>(p->nzb),
+                      ptr<int32_t>(p->nze), ptr<int64_t>(p->bprod), ptr<int64_t>(p->bslot), st);
+  tl_launches += 1;
+  launch_scan_i64(ptr<int64_t>(p->bprod), ptr<int64_t>(p->pool_off), max_blocks, scal + 0, ptr<int64_t>(p->scan_tmp), st);
+  launch_scan_i64(ptr<int64_t>(p->bslot), ptr<int64_t>(p->desc_off), max_blocks, scal + 1, ptr<int64_t>(p->scan_tmp), st);
+  tl_launches += 6;
+  k_put_i64<<<1, 1, 0, st>>>(scal + 2, nblocks_dev);
+  tl_launches += 1;
+  ACS_CUDA(cudaGetLastError());
+  if ((s = sync_read(p, scal, 3, st)) != ACSPGEMM_OK) return s;
+  const int64_t products = p->h_scal[0], slots = p->h_scal[1], nblocks = p->h_scal[2];
+  p->info.products = products;
+  p->info.nblocks = nblocks;
+  p->info.nsegments = nseg;
+  {
+    // segment boundaries for info (tiny copy)
+    int64_t segtab[MAX_SEGMENTS + 1];
+    ACS_CUDA(cudaMemcpy(segtab, p->seg.p, sizeof(int64_t) * (nseg + 1), cudaMemcpyDeviceToHost));
+    for (int i = 0; i <= nseg; ++i) p->info.segment_rows[i] = segtab[i];
+  }
+  const int64_t pool_bytes = products * (4 + vbytes);
+  if (p->opt.pool_limit_bytes && (size_t)pool_bytes > p->opt.pool_limit_bytes)
+    return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, "exact chunk-pool bound " + std::to_string(pool_bytes) +
+                                                   " B exceeds pool_limit_bytes");
+  ACS_ENSURE(p->pool_col, sizeof(int32_t) * products);
+  ACS_ENSURE(p->pool_val, (size_t)vbytes * products);
+  ACS_ENSURE(p->descs, sizeof(ChunkDesc) * slots);
+  ACS_ENSURE(p->row_count, sizeof(int32_t) * A->rows);
+  // scans later run over up to `slots` chunks / shared rows
+  ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * scan_tmp_elems(std::max<int64_t>(std::max(max_blocks, A->rows), slots) + 1));
+  p->info.pool_bytes = (int64_t)(p->pool_col.bytes + p->pool_val.bytes);
+  ACS_CUDA(cudaMemsetAsync(p->row_count.p, 0, sizeof(int32_t) * A->rows, st));
+
+  // ------------------------------------------------------------ ESC -----------
+  record(p, S_ESC, st);
+  EscArgs ea;
+  ea.A = Av;
+  ea.B = Bv;
+  ea.nblocks = (int32_t)nblocks;
+  ea.blk_nz_begin = ptr<int32_t>(p->nzb);
+  ea.blk_nz_end = ptr<int32_t>(p->nze);
+  ea.block_row_starts = ptr<int32_t>(p->brs);
+  ea.pool_off = ptr<int64_t>(p->pool_off);
+  ea.desc_off = ptr<int64_t>(p->desc_off);
+  ea.pool_col = ptr<int32_t>(p->pool_col);
+  ea.pool_val = p->pool_val.p;
+  ea.descs = ptr<ChunkDesc>(p->descs);
+  ea.nchunks = ptr<int32_t>(p->nchunks);
+  ea.used = ptr<int32_t>(p->bused);
+  ea.row_count = ptr<int32_t>(p->row_count);
+  launch_esc(ea, p->f64, st);
+  tl_launches += nblocks > 0 ? 1 : 0;
+  ACS_CUDA(cudaGetLastError());
+
+  // ------------------------------------------------------------ MCC -----------
+  record(p, S_MCC, st);
+  ACS_ENSURE(p->dense, sizeof(ChunkDesc) * slots);
+  ACS_ENSURE(p->sflag, sizeof(int32_t) * slots);
+  ACS_ENSURE(p->spos, sizeof(int64_t) * slots);
+  ACS_ENSURE(p->shared, sizeof(SharedRow) * slots);
+  launch_scan_i32(ptr<int32_t>(p->nchunks), ptr<int64_t>(p->chunk_base), nblocks, scal + 3, ptr<int64_t>(p->scan_tmp), st);
+  launch_scan_i32(ptr<int32_t>(p->bused), ptr<int64_t>(p->bused_scan), nblocks, scal + 5, ptr<int64_t>(p->scan_tmp), st);
+  tl_launches += 6;
+  MergeState ms;
+  ms.nblocks = (int32_t)nblocks;
+  ms.desc_off = ptr<int64_t>(p->desc_off);
+  ms.nchunks = ptr<int32_t>(p->nchunks);
+  ms.chunk_base = ptr<int64_t>(p->chunk_base);
+  ms.descs = ptr<ChunkDesc>(p->descs);
+  ms.dense = ptr<ChunkDesc>(p->dense);
+  ms.max_chunks = slots;
+  ms.total_chunks_dev = scal + 3;
+  ms.shared_flag = ptr<int32_t>(p->sflag);
+  ms.shared_pos = ptr<int64_t>(p->spos);
+  ms.shared = ptr<SharedRow>(p->shared);
+  ms.scan_tmp = ptr<int64_t>(p->scan_tmp);
+  launch_gather_chunks(ms, st);
+  launch_find_shared(ms, scal + 4, st);
+  tl_launches += 1 + (slots > 0 ? 5 : 0);
+  ACS_CUDA(cudaGetLastError());
+  if ((s = sync_read(p, scal + 3, 3, st)) != ACSPGEMM_OK) return s;
+  p->total_chunks = p->h_scal[0];
+  p->nshared = p->h_scal[1];
+  p->max_chunks = slots;
+  p->info.nchunks = p->total_chunks;
+  p->info.nshared = p->nshared;
+  p->info.chunk_elems = p->h_scal[2];
+  const int64_t nsh = p->nshared;
+  int64_t nmulti = 0, npath = 0, nsearch = 0, merge_total = 0, ngroups = 0;
+  if (nsh > 0) {
+    ACS_ENSURE(p->kflag, sizeof(int32_t) * nsh);
+    ACS_ENSURE(p->kpos, sizeof(int64_t) * nsh);
+    ACS_ENSURE(p->lmulti, sizeof(int32_t) * nsh);
+    ACS_ENSURE(p->lpath, sizeof(int32_t) * nsh);
+    ACS_ENSURE(p->lsearch, sizeof(int32_t) * nsh);
+    ACS_ENSURE(p->mtscan, sizeof(int64_t) * nsh);
+    ACS_ENSURE(p->mscan, sizeof(int64_t) * nsh);
+    ACS_ENSURE(p->group_of, sizeof(int32_t) * nsh);
+    MergeLists L;
+    L.nshared = nsh;
+    L.shared = ptr<SharedRow>(p->shared);
+    L.kind_flag = ptr<int32_t>(p->kflag);
+    L.kind_pos = ptr<int64_t>(p->kpos);
+    L.multi_idx = ptr<int32_t>(p->lmulti);
+    L.path_idx = ptr<int32_t>(p->lpath);
+    L.search_idx = ptr<int32_t>(p->lsearch);
+    L.counts_dev = scal + 8;
+    L.merge_total_scan = ptr<int64_t>(p->mtscan);
+    L.multi_scan = ptr<int64_t>(p->mscan);
+    L.group_of = ptr<int32_t>(p->group_of);
+    L.group_start = nullptr;
+    L.scan_tmp = ptr<int64_t>(p->scan_tmp);
+    launch_classify(L, st);
+    tl_launches += 3 * 5 + 1 + 3 + 1;
+    ACS_CUDA(cudaGetLastError());
+    if ((s = sync_read(p, scal + 8, 5, st)) != ACSPGEMM_OK) return s;
+    nmulti = p->h_scal[0];
+    npath = p->h_scal[1];
+    nsearch = p->h_scal[2];
+    merge_total = p->h_scal[4];
+    // Multi-Merge packing needs the multi totals: scan them over the multi list
+    if (nmulti > 0) {
+      // upper bound of groups from merge_total (multi totals <= merge_total)
+      int64_t gmax = 2 * ((merge_total + CAP - 1) / CAP) + 2;
+      ACS_ENSURE(p->gstart, sizeof(int32_t) * 2 * (gmax + 1));
+      L.group_start = ptr<int32_t>(p->gstart);
+      launch_multi_groups(L, nmulti, gmax, st);
+      tl_launches += 1 + 3 + 1 + 1;
+      ngroups = gmax;
+    }
+    ACS_ENSURE(p->merge_col, sizeof(int32_t) * merge_total);
+    ACS_ENSURE(p->merge_val, (size_t)vbytes * merge_total);
+    ACS_ENSURE(p->cur_first, sizeof(int32_t) * p->total_chunks);
+    ACS_ENSURE(p->cur_last, sizeof(int32_t) * p->total_chunks);
+    MergeArgs ma;
+    ma.dense = ptr<ChunkDesc>(p->dense);
+    ma.shared = ptr<SharedRow>(p->shared);
+    ma.group_start = ptr<int32_t>(p->gstart);
+    ma.multi_scan = ptr<int64_t>(p->mscan);
+    ma.ngroups = ngroups;
+    ma.pool_col = ptr<int32_t>(p->pool_col);
+    ma.pool_val = p->pool_val.p;
+    ma.merge_col = ptr<int32_t>(p->merge_col);
+    ma.merge_val = p->merge_val.p;
+    ma.cur_first = ptr<int32_t>(p->cur_first);
+    ma.cur_last = ptr<int32_t>(p->cur_last);
+    ma.row_count = ptr<int32_t>(p->row_count);
+    ma.error_flag = ptr<int32_t>(p->err);
+    record(p, S_MM, st);
+    ma.list = ptr<int32_t>(p->lmulti);
+    ma.nlist = nmulti;
+    if (nmulti > 0) { launch_multi_merge(ma, p->f64, st); tl_launches += 1; }
+    record(p, S_PM, st);
+    ma.list = ptr<int32_t>(p->lpath);
+    ma.nlist = npath;
+    if (npath > 0) { launch_path_merge(ma, p->f64, st); tl_launches += 1; }
+    record(p, S_SM, st);
+    ma.list = ptr<int32_t>(p->lsearch);
+    ma.nlist = nsearch;
+    if (nsearch > 0) { launch_search_merge(ma, p->f64, st); tl_launches += 1; }
+    ACS_CUDA(cudaGetLastError());
+  } else {
+    record(p, S_MM, st);
+    record(p, S_PM, st);
+    record(p, S_SM, st);
+  }
+  p->info.nmulti = nmulti;
+  p->info.npath = npath;
+  p->info.nsearch = nsearch;
+  p->info.nmulti_groups = ngroups;
+  p->info.merge_elems = merge_total;
+
+  // ------------------------------------------------------------ SCAN ----------
+  record(p, S_SCAN, st);
+  ACS_ENSURE(p->row_ptr, sizeof(int32_t) * (A->rows + 1));
+  launch_scan_rowptr(ptr<int32_t>(p->row_count), ptr<int32_t>(p->row_ptr), A->rows, scal + 16,
+                     ptr<int64_t>(p->scan_tmp), st);
+  tl_launches += 3;
+  ACS_CUDA(cudaGetLastError());
+  ACS_CUDA(cudaMemcpyAsync(p->h_scal, scal + 16, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+  ACS_CUDA(cudaMemcpyAsync(p->h_scal + 1, p->err.p, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  record(p, S_CC, st);
+  ACS_CUDA(cudaStreamSynchronize(st));
+  const int64_t nnz = p->h_scal[0];
+  const int32_t errflag = *reinterpret_cast<int32_t*>(p->h_scal + 1);
+  if (errflag) return set_err(ACSPGEMM_ERR_INTERNAL, "a shared row spans more chunks than one merge block handles");
+  if (nnz >= (int64_t(1) << 31)) return set_err(ACSPGEMM_ERR_INDEX_OVERFLOW, "nnz(C) >= 2^31");
+  p->nnz = nnz;
+  p->info.nnz_c = nnz;
+  p->info.helper_bytes = helper_bytes(p);
+  p->launches_sym = tl_launches - l0;
+  p->ready = true;
+  *nnz_c = nnz;
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t st) {
+  if (!p->ready) return set_err(ACSPGEMM_ERR_NOT_READY, "numeric called without a successful symbolic");
+  if (!C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C is NULL");
+  if (p->rows > 0 && !C->row_ptr) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C.row_ptr is NULL");
+  if (p->nnz > 0 && (!C->col_idx || !C->val)) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C.col_idx/val is NULL");
+  const long long l0 = tl_launches;
+  C->rows = p->rows;
+  C->cols = p->cols;
+  C->nnz = p->nnz;
+  if (p->empty) {
+    if (p->rows >= 0 && C->row_ptr) ACS_CUDA(cudaMemsetAsync(C->row_ptr, 0, sizeof(int32_t) * (p->rows + 1), st));
+    p->info.kernel_launches = p->launches_sym;
+    return ACSPGEMM_OK;
+  }
+  ACS_CUDA(cudaMemcpyAsync(C->row_ptr, p->row_ptr.p, sizeof(int32_t) * (p->rows + 1), cudaMemcpyDeviceToDevice, st));
+  record(p, S_CC, st);
+  CopyArgs ca;
+  ca.dense = ptr<ChunkDesc>(p->dense);
+  ca.total_chunks_dev = ptr<int64_t>(p->scal) + 3;
+  ca.max_chunks = p->total_chunks;
+  ca.shared = ptr<SharedRow>(p->shared);
+  ca.nshared = p->nshared;
+  ca.pool_col = ptr<int32_t>(p->pool_col);
+  ca.pool_val = p->pool_val.p;
+  ca.merge_col = ptr<int32_t>(p->merge_col);
+  ca.merge_val = p->merge_val.p;
+  ca.row_ptr = ptr<int32_t>(p->row_ptr);
+  ca.c_col = C->col_idx;
+  ca.c_val = C->val;
+  launch_copy(ca, p->f64, st);
+  if (p->total_chunks + p->nshared > 0) tl_launches += 1;
+  record(p, S_END, st);
+  ACS_CUDA(cudaGetLastError());
+  p->info.kernel_launches = p->launches_sym + (tl_launches - l0);
+  return ACSPGEMM_OK;
+}
+
+// ------------------------------------------------------------ debug kernels ------
+
+__global__ void k_debug_wd(const int32_t* lengths, int nentries, const int32_t* draws, int ndraws, int32_t* ares_out,
+                           int32_t* bres_out, int32_t* rem_out) {
+  __shared__ int wd[NPB + 1];
+  __shared__ int offsets[CAP_PAD];
+  __shared__ int scratch[40];
+  int len[NNZ_PER_THREAD];
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+    const int e = threadIdx.x * NNZ_PER_THREAD + j;
+    len[j] = e < nentries ? lengths[e] : 0;
+  }
+  wd_placework(len, wd, scratch);
+  int off = 0;
+  for (int d = 0; d < ndraws; ++d) {
+    const int consume = draws[d];
+    int ares[ITEMS], bres[ITEMS];
+    wd_receivework(consume, wd, offsets, scratch, ares, bres);
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+      const int c = i * THREADS + threadIdx.x;
+      if (c < consume) { ares_out[off + c] = ares[i]; bres_out[off + c] = bres[i]; }
+    }
+    for (int e = threadIdx.x; e < nentries; e += THREADS) rem_out[d * nentries + e] = wd[e + 1] - wd[e];
+    off += consume;
+    __syncthreads();
+  }
+}
+
+__global__ void k_debug_sort_compact(const int32_t* rows, const int32_t* cols, const double* vals, int n,
+                                     int32_t* orow, int32_t* ocol, double* oval, uint32_t* ostate) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  SortSmem<double>& S = *reinterpret_cast<SortSmem<double>*>(smem_raw);
+  const int tid = threadIdx.x;
+  int rmin = INT_MAX, rmax = INT_MIN, cmin = INT_MAX, cmax = INT_MIN;
+  for (int p = tid; p < n; p += THREADS) {
+    rmin = min(rmin, rows[p]); rmax = max(rmax, rows[p]);
+    cmin = min(cmin, cols[p]); cmax = max(cmax, cols[p]);
+  }
+  block_minmax4(rmin, rmax, cmin, cmax, S.scratch);
+  if (n == 0) return;
+  const int rowbits = bit_width_u64((uint64_t)(rmax - rmin));
+  const int colbits = bit_width_u64((uint64_t)((int64_t)cmax - cmin));
+  for (int p = tid; p < CAP; p += THREADS) {
+    if (p < n) {
+      const uint64_t key = ((uint64_t)(rows[p] - rmin) << colbits) | (uint64_t)(cols[p] - cmin);
+      S.words[pad32(p)] = (key << IDXBITS) | (uint64_t)p;
+      S.vals[p] = vals[p];
+    } else {
+      S.words[pad32(p)] = ~0ull;
+    }
+  }
+  __syncthreads();
+  uint64_t k[ITEMS];
+  double ev[ITEMS];
+  load_and_sort<uint64_t, double>(S, rowbits + colbits, k);
+  const ScanCtx<uint64_t, double> ctx = compaction_prepare<uint64_t, double>(S, k, n, colbits, ev);
+  const uint64_t colmask = colbits ? ((1ull << colbits) - 1) : 0;
+  compaction_emit<uint64_t, double, true>(k, ev, n, colbits, ctx,
+                                          [&](int idx, uint64_t key, double val, uint32_t state, bool) {
+    orow[idx] = rmin + (int)(key >> colbits);
+    ocol[idx] = cmin + (int)(key & colmask);
+    oval[idx] = val;
+    ostate[idx] = state;
+  });
+}
+
+template <typename P>
+struct Scratch {
+  P* d = nullptr;
+  ~Scratch() { if (d) cudaFree(d); }
+};
+
+}  // namespace
+
+// ======================================================================= C ABI ====
+
+extern "C" {
+
+void acspgemm_options_default(acspgemm_options* opt) {
+  if (!opt) return;
+  opt->pool_limit_bytes = 0;
+  opt->validate_inputs = 0;
+  opt->collect_stage_times = 0;
+  opt->num_segments = DEFAULT_SEGMENTS;
+}
+
+acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options* opt) {
+  if (!plan) return set_err(ACSPGEMM_ERR_INVALID_ARG, "plan is NULL");
+  acspgemm_plan p = new (std::nothrow) acspgemm_plan_s();
+  if (!p) return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, "host allocation");
+  acspgemm_options_default(&p->opt);
+  if (opt) p->opt = *opt;
+  if (p->opt.num_segments <= 0) p->opt.num_segments = DEFAULT_SEGMENTS;
+  if (p->opt.num_segments > MAX_SEGMENTS) {
+    delete p;
+    return set_err(ACSPGEMM_ERR_INVALID_ARG, "num_segments > 64");
+  }
+  std::memset(&p->info, 0, sizeof(p->info));
+  cudaError_t e = cudaHostAlloc(&p->h_scal, sizeof(int64_t) * 32, cudaHostAllocDefault);
+  if (e != cudaSuccess) {
+    delete p;
+    return set_err(ACSPGEMM_ERR_CUDA, std::string("cudaHostAlloc: ") + cudaGetErrorString(e));
+  }
+  p->ev_ok = true;
+  for (int i = 0; i < NSTAGE_EV; ++i)
+    if (cudaEventCreate(&p->ev[i]) != cudaSuccess) p->ev_ok = false;
+  *plan = p;
+  return ACSPGEMM_OK;
+}
+
+void acspgemm_plan_destroy(acspgemm_plan p) {
+  if (!p) return;
+  cudaDeviceSynchronize();
+  DevBuf* bs[] = {&p->seg, &p->seg_rows, &p->scal, &p->brs, &p->nzb, &p->nze, &p->bprod, &p->bslot,
+                  &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->pool_col, &p->pool_val,
+                  &p->descs, &p->dense, &p->sflag, &p->spos, &p->shared, &p->row_count, &p->row_ptr,
+                  &p->scan_tmp, &p->kflag, &p->kpos, &p->lmulti, &p->lpath, &p->lsearch, &p->mscan,
+                  &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
+                  &p->cur_last, &p->err, &p->bused, &p->bused_scan};
+  for (DevBuf* b : bs) free_buf(*b);
+  if (p->h_scal) cudaFreeHost(p->h_scal);
+  if (p->ev_ok)
+    for (int i = 0; i < NSTAGE_EV; ++i) cudaEventDestroy(p->ev[i]);
+  delete p;
+}
+
+acspgemm_status acspgemm_set_segments(acspgemm_plan p, int nseg, const int64_t* rows_host) {
+  if (!p) return set_err(ACSPGEMM_ERR_INVALID_ARG, "plan is NULL");
+  if (nseg == 0) { p->nseg_explicit = 0; return ACSPGEMM_OK; }
+  if (nseg < 0 || nseg > MAX_SEGMENTS || !rows_host) return set_err(ACSPGEMM_ERR_INVALID_ARG, "bad segments");
+  if (rows_host[0] != 0) return set_err(ACSPGEMM_ERR_INVALID_ARG, "segments must start at row 0");
+  for (int i = 0; i < nseg; ++i)
+    if (rows_host[i + 1] < rows_host[i]) return set_err(ACSPGEMM_ERR_INVALID_ARG, "segments must be non-decreasing");
+  for (int i = 0; i <= nseg; ++i) p->seg_rows_explicit[i] = rows_host[i];
+  p->nseg_explicit = nseg;
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status acspgemm_canonical_segments(const acspgemm_csr_in* A, int nseg, int64_t* rows_host, void* stream) {
+  acspgemm_status s = check_in(A, "A");
+  if (s != ACSPGEMM_OK) return s;
+  if (nseg < 1 || nseg > MAX_SEGMENTS || !rows_host) return set_err(ACSPGEMM_ERR_INVALID_ARG, "bad nseg");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  if (A->rows == 0) {
+    for (int i = 0; i <= nseg; ++i) rows_host[i] = 0;
+    return ACSPGEMM_OK;
+  }
+  Scratch<int64_t> seg;
+  ACS_CUDA(cudaMalloc(&seg.d, sizeof(int64_t) * (3 * (MAX_SEGMENTS + 1) + 2)));
+  const CsrView Av{A->rows, A->cols, A->row_ptr, A->col_idx, A->val};
+  launch_segments(Av, nseg, nullptr, seg.d, reinterpret_cast<int32_t*>(seg.d + 3 * (MAX_SEGMENTS + 1)), st);
+  ACS_CUDA(cudaGetLastError());
+  ACS_CUDA(cudaMemcpyAsync(rows_host, seg.d, sizeof(int64_t) * (nseg + 1), cudaMemcpyDeviceToHost, st));
+  ACS_CUDA(cudaStreamSynchronize(st));
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status acspgemm_symbolic(acspgemm_plan p, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
+                                  acspgemm_dtype dtype, void* stream, int64_t* nnz_c) {
+  if (!p) return set_err(ACSPGEMM_ERR_INVALID_ARG, "plan is NULL");
+  return symbolic_impl(p, A, B, dtype, reinterpret_cast<cudaStream_t>(stream), nnz_c);
+}
+
+acspgemm_status acspgemm_numeric(acspgemm_plan p, acspgemm_csr_out* C, void* stream) {
+  if (!p) return set_err(ACSPGEMM_ERR_INVALID_ARG, "plan is NULL");
+  return numeric_impl(p, C, reinterpret_cast<cudaStream_t>(stream));
+}
+
+acspgemm_status acspgemm_multiply(const acspgemm_csr_in* A, const acspgemm_csr_in* B, acspgemm_csr_out* C,
+                                  void* stream, acspgemm_dtype dtype) {
+  if (!C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C is NULL");
+  acspgemm_plan p = nullptr;
+  acspgemm_status s = acspgemm_plan_create(&p, nullptr);
+  if (s != ACSPGEMM_OK) return s;
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  int64_t nnz = 0;
+  s = acspgemm_symbolic(p, A, B, dtype, stream, &nnz);
+  if (s == ACSPGEMM_OK) {
+    const size_t vb = dtype == ACSPGEMM_F64 ? 8 : 4;
+    C->row_ptr = nullptr; C->col_idx = nullptr; C->val = nullptr;
+    cudaError_t e = cudaMallocAsync((void**)&C->row_ptr, sizeof(int32_t) * (A->rows + 1), st);
+    if (e == cudaSuccess) e = cudaMallocAsync((void**)&C->col_idx, sizeof(int32_t) * (nnz > 0 ? nnz : 1), st);
+    if (e == cudaSuccess) e = cudaMallocAsync(&C->val, vb * (nnz > 0 ? nnz : 1), st);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      acspgemm_free_csr(C, stream);
+      s = set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, std::string("cudaMallocAsync: ") + cudaGetErrorString(e));
+    } else {
+      s = acspgemm_numeric(p, C, stream);
+    }
+  }
+  if (s == ACSPGEMM_OK) cudaStreamSynchronize(st);
+  acspgemm_plan_destroy(p);
+  return s;
+}
+
+acspgemm_status acspgemm_free_csr(acspgemm_csr_out* C, void* stream) {
+  if (!C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C is NULL");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  if (C->row_ptr) cudaFreeAsync(C->row_ptr, st);
+  if (C->col_idx) cudaFreeAsync(C->col_idx, st);
+  if (C->val) cudaFreeAsync(C->val, st);
+  C->row_ptr = nullptr; C->col_idx = nullptr; C->val = nullptr;
+  ACS_CUDA(cudaGetLastError());
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status acspgemm_stage_times(acspgemm_plan p, float* ms_out, int n) {
+  if (!p || !ms_out) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
+  if (!p->opt.collect_stage_times || !p->ev_ok) return set_err(ACSPGEMM_ERR_NOT_READY, "stage times not collected");
+  if (p->empty) {
+    for (int i = 0; i < n && i < 8; ++i) ms_out[i] = 0.f;
+    return ACSPGEMM_OK;
+  }
+  ACS_CUDA(cudaEventSynchronize(p->ev[S_END]));
+  for (int i = 0; i < n && i < 8; ++i) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, p->ev[i], p->ev[i + 1]) != cudaSuccess) { cudaGetLastError(); ms = -1.f; }
+    ms_out[i] = ms;
+  }
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status acspgemm_plan_info(acspgemm_plan p, acspgemm_info* info) {
+  if (!p || !info) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
+  *info = p->info;
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status acspgemm_block_row_starts(acspgemm_plan p, int32_t* host_out, int64_t n) {
+  if (!p || (!host_out && n > 0)) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
+  if (!p->ready) return set_err(ACSPGEMM_ERR_NOT_READY, "no symbolic pass");
+  if (n > p->info.nblocks) n = p->info.nblocks;
+  if (n <= 0) return ACSPGEMM_OK;
+  ACS_CUDA(cudaMemcpy(host_out, p->brs.p, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+  return ACSPGEMM_OK;
+}
+
+double acspgemm_pool_estimate_bytes(int64_t nA, int64_t nnzA, int64_t nB, int64_t mB, int64_t nnzB,
+                                    int value_bytes) {
+  double S = 0.0;
+  if (nA > 0 && nB > 0 && mB > 0 && nnzA > 0 && nnzB > 0) {
+    const double a = (double)nnzA / (double)nA;
+    const double b = (double)nnzB / (double)nB;
+    const double pb = b / (double)mB;
+    S = pb < 1.0 ? (double)nA * b * (-std::expm1(a * std::log1p(-pb))) / pb : (double)nA * b;
+  }
+  const double bytes = S * (4.0 + value_bytes) * 1.2;
+  return bytes > 100e6 ? bytes : 100e6;
+}
+
+acspgemm_status acspgemm_debug_work_distribution(const int32_t* lengths, int nentries, const int32_t* draws,
+                                                 int ndraws, int32_t* ares, int32_t* bres, int32_t* remaining) {
+  if (nentries < 0 || nentries > NPB || ndraws < 0 || (!lengths && nentries) || (!draws && ndraws))
+    return set_err(ACSPGEMM_ERR_INVALID_ARG, "bad arguments");
+  int64_t total_len = 0, total_draw = 0;
+  for (int i = 0; i < nentries; ++i) total_len += lengths[i];
+  for (int d = 0; d < ndraws; ++d) {
+    if (draws[d] < 0 || draws[d] > CAP) return set_err(ACSPGEMM_ERR_INVALID_ARG, "draw > CAP");
+    total_draw += draws[d];
+  }
+  if (total_draw > total_len) return set_err(ACSPGEMM_ERR_INVALID_ARG, "draws exceed the work");
+  Scratch<int32_t> dl, dd, da, db, dr;
+  ACS_CUDA(cudaMalloc(&dl.d, sizeof(int32_t) * (nentries + 1)));
+  ACS_CUDA(cudaMalloc(&dd.d, sizeof(int32_t) * (ndraws + 1)));
+  ACS_CUDA(cudaMalloc(&da.d, sizeof(int32_t) * (total_draw + 1)));
+  ACS_CUDA(cudaMalloc(&db.d, sizeof(int32_t) * (total_draw + 1)));
+  ACS_CUDA(cudaMalloc(&dr.d, sizeof(int32_t) * ((int64_t)ndraws * nentries + 1)));
+  if (nentries) ACS_CUDA(cudaMemcpy(dl.d, lengths, sizeof(int32_t) * nentries, cudaMemcpyHostToDevice));
+  if (ndraws) ACS_CUDA(cudaMemcpy(dd.d, draws, sizeof(int32_t) * ndraws, cudaMemcpyHostToDevice));
+  k_debug_wd<<<1, THREADS>>>(dl.d, nentries, dd.d, ndraws, da.d, db.d, dr.d);
+  ACS_CUDA(cudaGetLastError());
+  ACS_CUDA(cudaDeviceSynchronize());
+  if (total_draw) {
+    ACS_CUDA(cudaMemcpy(ares, da.d, sizeof(int32_t) * total_draw, cudaMemcpyDeviceToHost));
+    ACS_CUDA(cudaMemcpy(bres, db.d, sizeof(int32_t) * total_draw, cudaMemcpyDeviceToHost));
+  }
+  if ((int64_t)ndraws * nentries)
+    ACS_CUDA(cudaMemcpy(remaining, dr.d, sizeof(int32_t) * ndraws * nentries, cudaMemcpyDeviceToHost));
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status acspgemm_debug_sort_compact(const int32_t* rows, const int32_t* cols, const double* vals, int n,
+                                            int32_t* out_rows, int32_t* out_cols, double* out_vals,
+                                            uint32_t* out_state) {
+  if (n < 0 || n > CAP) return set_err(ACSPGEMM_ERR_INVALID_ARG, "n must be in [0, CAP]");
+  if (n == 0) return ACSPGEMM_OK;
+  Scratch<int32_t> dr, dc, orow, ocol;
+  Scratch<double> dv, oval;
+  Scratch<uint32_t> ost;
+  ACS_CUDA(cudaMalloc(&dr.d, sizeof(int32_t) * n));
+  ACS_CUDA(cudaMalloc(&dc.d, sizeof(int32_t) * n));
+  ACS_CUDA(cudaMalloc(&dv.d, sizeof(double) * n));
+  ACS_CUDA(cudaMalloc(&orow.d, sizeof(int32_t) * n));
+  ACS_CUDA(cudaMalloc(&ocol.d, sizeof(int32_t) * n));
+  ACS_CUDA(cudaMalloc(&oval.d, sizeof(double) * n));
+  ACS_CUDA(cudaMalloc(&ost.d, sizeof(uint32_t) * n));
+  ACS_CUDA(cudaMemcpy(dr.d, rows, sizeof(int32_t) * n, cudaMemcpyHostToDevice));
+  ACS_CUDA(cudaMemcpy(dc.d, cols, sizeof(int32_t) * n, cudaMemcpyHostToDevice));
+  ACS_CUDA(cudaMemcpy(dv.d, vals, sizeof(double) * n, cudaMemcpyHostToDevice));
+  const size_t smem = sizeof(SortSmem<double>);
+  ACS_CUDA(cudaFuncSetAttribute(k_debug_sort_compact, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  k_debug_sort_compact<<<1, THREADS, smem>>>(dr.d, dc.d, dv.d, n, orow.d, ocol.d, oval.d, ost.d);
+  ACS_CUDA(cudaGetLastError());
+  ACS_CUDA(cudaDeviceSynchronize());
+  ACS_CUDA(cudaMemcpy(out_rows, orow.d, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+  ACS_CUDA(cudaMemcpy(out_cols, ocol.d, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+  ACS_CUDA(cudaMemcpy(out_vals, oval.d, sizeof(double) * n, cudaMemcpyDeviceToHost));
+  ACS_CUDA(cudaMemcpy(out_state, ost.d, sizeof(uint32_t) * n, cudaMemcpyDeviceToHost));
+  return ACSPGEMM_OK;
+}
+
+int acspgemm_const(int id) {
+  switch (id) {
+    case 0: return NPB;
+    case 1: return THREADS;
+    case 2: return ITEMS;
+    case 3: return CAP;
+    case 4: return KEEP;
+    case 5: return RADIX_BITS;
+    case 6: return DEFAULT_SEGMENTS;
+    case 7: return PATH_MAX_CHUNKS;
+    default: return -1;
+  }
+}
+
+const char* acspgemm_status_string(acspgemm_status s) {
+  switch (s) {
+    case ACSPGEMM_OK: return "ok";
+    case ACSPGEMM_ERR_INVALID_ARG: return "invalid argument";
+    case ACSPGEMM_ERR_DIM_MISMATCH: return "dimension mismatch";
+    case ACSPGEMM_ERR_INDEX_OVERFLOW: return "index overflow";
+    case ACSPGEMM_ERR_OUT_OF_MEMORY: return "out of memory";
+    case ACSPGEMM_ERR_CUDA: return "cuda error";
+    case ACSPGEMM_ERR_NOT_READY: return "not ready";
+    case ACSPGEMM_ERR_INTERNAL: return "internal limit";
+  }
+  return "unknown";
+}
+
+const char* acspgemm_last_error(void) { return tl_err.c_str(); }
+
+int acspgemm_abi_version(void) { return ACSPGEMM_ABI_VERSION; }
+
+}  // extern "C"
