@@ -28,7 +28,10 @@ constexpr int NPB = 512;                     // NNZ_PER_BLOCK (Alg. 1, Alg. 2; L
 constexpr int NNZ_PER_THREAD = NPB / THREADS;// A entries per thread
 constexpr int KEEP_PER_THREAD = 4;           // "keeps up to 4 elements per thread" (L556)
 constexpr int KEEP = KEEP_PER_THREAD * THREADS; // max kept elements of the last row
-constexpr int RADIX_BITS = 5;                // digit width of one radix-sort pass
+#ifndef ACS_RADIX_BITS
+#define ACS_RADIX_BITS 5
+#endif
+constexpr int RADIX_BITS = ACS_RADIX_BITS;   // digit width of one radix-sort pass
 constexpr int DEFAULT_SEGMENTS = 8;          // canonical segments
 constexpr int MAX_SEGMENTS = 64;
 constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)

@@ -103,16 +103,19 @@ __device__ __forceinline__ void wd_receivework(int consume, int* wd, int* offset
 // radix sort keeps equal keys in position order, i.e. the expansion order (kept
 // elements first, then products by A entry) that the paper's stable sort preserves
 // for bit-stable sums (L198).  Ranking: per-thread 16-bit digit counters packed two per
-// word (RADIX_BITS = 5 -> 32 digits = 16 counter lanes x 2 halves), a raking exclusive
+// word (RADIX_BITS = b -> 2^b digits = 2^(b-1) counter lanes x 2 halves), a raking exclusive
 // scan over (lane, thread) order, a scatter through shared memory.  Five barriers per
 // pass.  Words live at pad32(index).
 // =====================================================================
 
-constexpr int CNT_LANES = 16;
-constexpr int LANE_STRIDE = THREADS + THREADS / 32;         // padded words per counter lane
+constexpr int CNT_LANES = 1 << (RADIX_BITS - 1);               // two 16-bit digits per word
+#ifndef ACS_LANE_STRIDE
+#define ACS_LANE_STRIDE (ACS_THREADS + ACS_THREADS / 32)
+#endif
+constexpr int LANE_STRIDE = ACS_LANE_STRIDE;                // padded words per counter lane
 constexpr int CNT_PADDED = CNT_LANES * LANE_STRIDE;
 constexpr int RAKE = CNT_LANES;                             // words per thread in the raking scan
-static_assert(RADIX_BITS <= 5, "two 16-bit halves x 16 lanes");
+static_assert(RADIX_BITS >= 2 && RADIX_BITS <= 6, "two 16-bit halves x CNT_LANES lanes");
 static_assert(THREADS % 32 == 0 && RAKE <= 32 && 32 % RAKE == 0, "raking layout");
 static_assert(ITEMS <= 32 && 32 % ITEMS == 0, "blocked items must not straddle padding");
 
@@ -122,7 +125,10 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
   const int tid = threadIdx.x, lane = lane_id(), w = warp_id();
   uint16_t* c16 = reinterpret_cast<uint16_t*>(s_cnt);
   const int tb2 = 2 * (tid + (tid >> 5));                   // my column in every counter lane
-  const int seg0 = pad32(tid * RAKE);                       // my raking segment (contiguous)
+  // my raking segment: logical counter words [tid*RAKE, (tid+1)*RAKE) = lane L, threads
+  // t0 .. t0+RAKE-1 (contiguous: RAKE divides 32)
+  const int t0 = (tid * RAKE) % THREADS;
+  const int seg0 = ((tid * RAKE) / THREADS) * LANE_STRIDE + t0 + (t0 >> 5);
   const int bb = pad32(tid * ITEMS);                        // my blocked items (contiguous)
   if (begin_bit >= end_bit) return;
 #pragma unroll
@@ -136,7 +142,7 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
       const uint32_t d = (uint32_t)(k[i] >> bit) & mask;
-      cidx[i] = (int)(d & 15u) * (2 * LANE_STRIDE) + (int)(d >> 4) + tb2;
+      cidx[i] = (int)(d & (CNT_LANES - 1)) * (2 * LANE_STRIDE) + (int)(d >> (RADIX_BITS - 1)) + tb2;
       pre[i] = c16[cidx[i]];
       c16[cidx[i]] = (uint16_t)(pre[i] + 1u);
     }
@@ -162,7 +168,7 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
     const uint32_t grand = __shfl_sync(0xffffffffu, wt, THREADS / 32 - 1);
     uint32_t wpre = __shfl_up_sync(0xffffffffu, wt, 1);
     wpre = __shfl_sync(0xffffffffu, lane == 0 ? 0u : wpre, w);
-    // digits 16..31 (high halves) follow all of 0..15 (low halves)
+    // digits in the high halves follow all digits in the low halves
     uint32_t run = wpre + inc - sum + ((grand & 0xFFFFu) << 16);
 #pragma unroll
     for (int j = 0; j < RAKE; ++j) { const uint32_t v = seg[j]; s_cnt[seg0 + j] = run; run += v; }
