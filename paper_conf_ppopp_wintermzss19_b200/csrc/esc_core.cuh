@@ -104,31 +104,41 @@ __device__ __forceinline__ void wd_receivework(int consume, int* wd, int* offset
 // elements first, then products by A entry) that the paper's stable sort preserves
 // for bit-stable sums (L198).  Ranking: per-thread 16-bit digit counters packed two per
 // word (RADIX_BITS = b -> 2^b digits = 2^(b-1) counter lanes x 2 halves), a raking exclusive
-// scan over (lane, thread) order, a scatter through shared memory.  Five barriers per
-// pass.  Words live at pad32(index).
+// scan over (lane, virtual thread) order, a scatter through shared memory.  Five
+// barriers per pass.  Words live at pad32(index).
 // =====================================================================
 
 constexpr int CNT_LANES = 1 << (RADIX_BITS - 1);               // two 16-bit digits per word
+// Each thread counts its ITEMS keys as VT "virtual threads" of ITEMS/VT consecutive keys
+// with separate counter columns: the VT read-increment-write chains are independent, so
+// their shared-memory latencies overlap; the (lane, virtual thread) scan order keeps the
+// ranking stable because virtual thread tid*VT + v holds keys tid*ITEMS + v*ITEMS/VT ...
+#ifndef ACS_VT
+#define ACS_VT 1
+#endif
+constexpr int VT = ACS_VT;
+constexpr int VTHREADS = THREADS * VT;
 #ifndef ACS_LANE_STRIDE
-#define ACS_LANE_STRIDE (ACS_THREADS + ACS_THREADS / 32)
+#define ACS_LANE_STRIDE (ACS_THREADS * ACS_VT + ACS_THREADS * ACS_VT / 32)
 #endif
 constexpr int LANE_STRIDE = ACS_LANE_STRIDE;                // padded words per counter lane
 constexpr int CNT_PADDED = CNT_LANES * LANE_STRIDE;
-constexpr int RAKE = CNT_LANES;                             // words per thread in the raking scan
+constexpr int RAKE = CNT_LANES * VT;                        // words per thread in the raking scan
 static_assert(RADIX_BITS >= 2 && RADIX_BITS <= 6, "two 16-bit halves x CNT_LANES lanes");
-static_assert(THREADS % 32 == 0 && RAKE <= 32 && 32 % RAKE == 0, "raking layout");
+static_assert(VTHREADS % 32 == 0 && RAKE <= 32 && 32 % RAKE == 0, "raking layout");
 static_assert(ITEMS <= 32 && 32 % ITEMS == 0, "blocked items must not straddle padding");
+static_assert(ITEMS % VT == 0, "virtual threads split the items evenly");
 
 template <typename Word>
 __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words, uint32_t* s_cnt,
                                                  uint32_t* s_warp, int begin_bit, int end_bit) {
+  constexpr int IPV = ITEMS / VT;                           // items per virtual thread
   const int tid = threadIdx.x, lane = lane_id(), w = warp_id();
   uint16_t* c16 = reinterpret_cast<uint16_t*>(s_cnt);
-  const int tb2 = 2 * (tid + (tid >> 5));                   // my column in every counter lane
-  // my raking segment: logical counter words [tid*RAKE, (tid+1)*RAKE) = lane L, threads
-  // t0 .. t0+RAKE-1 (contiguous: RAKE divides 32)
-  const int t0 = (tid * RAKE) % THREADS;
-  const int seg0 = ((tid * RAKE) / THREADS) * LANE_STRIDE + t0 + (t0 >> 5);
+  // my raking segment: logical counter words [tid*RAKE, (tid+1)*RAKE) = lane L, virtual
+  // threads v0 .. v0+RAKE-1 (contiguous: RAKE divides 32)
+  const int v0 = (tid * RAKE) % VTHREADS;
+  const int seg0 = ((tid * RAKE) / VTHREADS) * LANE_STRIDE + v0 + (v0 >> 5);
   const int bb = pad32(tid * ITEMS);                        // my blocked items (contiguous)
   if (begin_bit >= end_bit) return;
 #pragma unroll
@@ -140,11 +150,16 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
     int cidx[ITEMS];
     uint32_t pre[ITEMS];
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-      const uint32_t d = (uint32_t)(k[i] >> bit) & mask;
-      cidx[i] = (int)(d & (CNT_LANES - 1)) * (2 * LANE_STRIDE) + (int)(d >> (RADIX_BITS - 1)) + tb2;
-      pre[i] = c16[cidx[i]];
-      c16[cidx[i]] = (uint16_t)(pre[i] + 1u);
+    for (int q = 0; q < IPV; ++q) {
+#pragma unroll
+      for (int v = 0; v < VT; ++v) {
+        const int i = v * IPV + q;
+        const int vt = tid * VT + v;
+        const uint32_t d = (uint32_t)(k[i] >> bit) & mask;
+        cidx[i] = (int)(d & (CNT_LANES - 1)) * (2 * LANE_STRIDE) + (int)(d >> (RADIX_BITS - 1)) + 2 * (vt + (vt >> 5));
+        pre[i] = c16[cidx[i]];
+        c16[cidx[i]] = (uint16_t)(pre[i] + 1u);
+      }
     }
     __syncthreads();
     uint32_t seg[RAKE];
