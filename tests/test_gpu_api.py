@@ -1,0 +1,138 @@
+"""GPU tests of the C-ABI behaviour beyond parity: error statuses, plan reuse, streams,
+stage times, IEEE special values, empty inputs."""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth import CSR, from_coo, poisson2d_5pt, poisson3d_27pt, power_law_csr, random_csr
+
+pytestmark = pytest.mark.gpu
+
+
+def pkg():
+    import paper_conf_ppopp_wintermzss19_b200 as p
+    return p
+
+
+def dev(M, dt=np.float64):
+    return pkg().DeviceCSR.from_host(M, "cuda", dt)
+
+
+def check(C, A, B, tol=1e-12):
+    rp, col, val = C.to_numpy()
+    ref = oracle.gustavson(A, B)
+    assert (rp == ref.row_ptr).all() and (col == ref.col).all()
+    assert (np.abs(val.astype(np.float64) - ref.val) <= tol * ref.absval).all()
+
+
+def test_pool_limit_out_of_memory_then_recover(cuda_available):
+    p = pkg()
+    A = poisson3d_27pt(12)
+    dA = dev(A)
+    plan = p.Plan(pool_limit_bytes=1000)
+    with pytest.raises(p.AcspgemmError) as ei:
+        plan.multiply(dA, dA)
+    assert ei.value.status == 4                      # ACSPGEMM_ERR_OUT_OF_MEMORY
+    plan.close()
+    plan = p.Plan()                                  # a fresh plan works
+    check(plan.multiply(dA, dA), A, A)
+
+
+def test_numeric_before_symbolic_is_not_ready(cuda_available):
+    p = pkg()
+    plan = p.Plan()
+    t = torch.zeros(4, dtype=torch.int32, device="cuda")
+    v = torch.zeros(4, dtype=torch.float64, device="cuda")
+    with pytest.raises(p.AcspgemmError) as ei:
+        plan.numeric(t, t, v)
+    assert ei.value.status == 6                      # ACSPGEMM_ERR_NOT_READY
+
+
+def test_plan_reuse_grow_and_shrink(cuda_available):
+    p = pkg()
+    plan = p.Plan()
+    for A in (random_csr(50, 40, 0.1, seed=1), poisson3d_27pt(14), random_csr(300, 300, 0.02, seed=2),
+              power_law_csr(2000, 2000, 10, 1.3, 800, seed=3), poisson2d_5pt(8)):
+        B = A if A.rows == A.cols else random_csr(A.cols, 30, 0.2, seed=4)
+        check(plan.multiply(dev(A), dev(B)), A, B)
+
+
+def test_stage_times(cuda_available):
+    p = pkg()
+    A = power_law_csr(3000, 3000, 12, 1.2, 1500, seed=7)
+    plan = p.Plan(stage_times=True)
+    plan.multiply(dev(A), dev(A))
+    torch.cuda.synchronize()
+    st = plan.stage_times()
+    assert list(st) == list(p.STAGES)
+    assert all(v >= 0 for v in st.values()) and st["ESC"] > 0
+
+
+def test_two_plans_two_streams(cuda_available):
+    p = pkg()
+    A1, A2 = poisson3d_27pt(16), power_law_csr(4000, 4000, 10, 1.3, 1000, seed=11)
+    d1, d2 = dev(A1), dev(A2)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    p1, p2 = p.Plan(), p.Plan()
+    torch.cuda.synchronize()
+    with torch.cuda.stream(s1):
+        C1 = p1.multiply(d1, d1, s1)
+    with torch.cuda.stream(s2):
+        C2 = p2.multiply(d2, d2, s2)
+    torch.cuda.synchronize()
+    check(C1, A1, A1)
+    check(C2, A2, A2)
+
+
+def test_ieee_special_values(cuda_available):
+    """NaN and Inf propagate (no fast-math, reading R22): entries whose sum involves a
+    NaN are NaN, Inf·0 gives NaN, finite entries match the oracle."""
+    A = from_coo(3, 3, [0, 0, 1, 2], [0, 1, 1, 2], np.array([np.nan, 1.0, np.inf, 2.0]))
+    B = from_coo(3, 3, [0, 1, 1, 2], [0, 0, 2, 2], np.array([1.0, 3.0, 0.0, 5.0]))
+    C = pkg().multiply(dev(A), dev(B))
+    rp, col, val = C.to_numpy()
+    ref = oracle.gustavson(A, B)
+    assert (rp == ref.row_ptr).all() and (col == ref.col).all()
+    for g, r in zip(val, ref.val):
+        assert (math.isnan(g) and math.isnan(r)) or g == r
+
+
+def test_empty_inputs(cuda_available):
+    p = pkg()
+    Z = CSR(0, 5, np.zeros(1, np.int32), np.zeros(0, np.int32), np.zeros(0))
+    B = random_csr(5, 6, 0.5, seed=1)
+    C = p.multiply(dev(Z), dev(B))
+    assert C.rows == 0 and C.nnz == 0
+    Zr = random_csr(7, 5, 0.0, seed=2)
+    C = p.multiply(dev(Zr), dev(B))
+    rp, _, _ = C.to_numpy()
+    assert C.nnz == 0 and (rp == 0).all() and rp.shape[0] == 8
+    rp, col, val = p.multiply_lib_alloc(dev(Zr), dev(B))
+    assert rp.shape[0] == 8 and (rp == 0).all() and col.size == 0
+
+
+def test_fp32_accumulates_in_fp32(cuda_available):
+    """fp32 inputs accumulate in fp32 (reading R14): a row whose exact sum needs more than
+    24 bits differs from the fp64 oracle by at most the fp32 tolerance."""
+    n = 3000
+    A = from_coo(1, n, np.zeros(n), np.arange(n), np.full(n, 1.0 + 2.0 ** -20))
+    B = from_coo(n, 1, np.arange(n), np.zeros(n), np.full(n, 1.0 + 2.0 ** -21))
+    C = pkg().multiply(dev(A, np.float32), dev(B, np.float32))
+    _, _, val = C.to_numpy()
+    ref = oracle.gustavson(A.astype(np.float32), B.astype(np.float32))
+    assert val.dtype == np.float32
+    assert abs(float(val[0]) - ref.val[0]) <= 1e-5 * ref.absval[0]
+
+
+def test_binding_argument_checks(cuda_available):
+    p = pkg()
+    A = dev(random_csr(5, 5, 0.5, seed=3))
+    Af = dev(random_csr(5, 5, 0.5, seed=3), np.float32)
+    with pytest.raises(TypeError):
+        p.multiply(A, Af)
+    cpuA = p.DeviceCSR(A.rows, A.cols, A.row_ptr.cpu(), A.col.cpu(), A.val.cpu())
+    with pytest.raises(ValueError):
+        p.multiply(cpuA, cpuA)
