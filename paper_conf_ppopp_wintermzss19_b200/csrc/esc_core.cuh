@@ -118,8 +118,19 @@ constexpr int CNT_LANES = 1 << (RADIX_BITS - 1);               // two 16-bit dig
 #endif
 constexpr int VT = ACS_VT;
 constexpr int VTHREADS = THREADS * VT;
+// ACS_ROT_RAKE: counter lanes without padding (LANE_STRIDE = VTHREADS, a multiple of 32)
+// make the counting accesses bank-conflict free for any digits; the raking scan then
+// reads its 16-word segment in a per-thread rotated order (conflict free as well) and
+// undoes the rotation arithmetically.
+#ifndef ACS_ROT_RAKE
+#define ACS_ROT_RAKE 0
+#endif
 #ifndef ACS_LANE_STRIDE
+#if ACS_ROT_RAKE
+#define ACS_LANE_STRIDE (ACS_THREADS * ACS_VT)
+#else
 #define ACS_LANE_STRIDE (ACS_THREADS * ACS_VT + ACS_THREADS * ACS_VT / 32)
+#endif
 #endif
 constexpr int LANE_STRIDE = ACS_LANE_STRIDE;                // padded words per counter lane
 constexpr int CNT_PADDED = CNT_LANES * LANE_STRIDE;
@@ -138,11 +149,21 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
   // my raking segment: logical counter words [tid*RAKE, (tid+1)*RAKE) = lane L, virtual
   // threads v0 .. v0+RAKE-1 (contiguous: RAKE divides 32)
   const int v0 = (tid * RAKE) % VTHREADS;
+#if ACS_ROT_RAKE
+  static_assert(RAKE == 16 && VT == 1, "rotated raking layout");
+  const int seg0 = ((tid * RAKE) / VTHREADS) * LANE_STRIDE + v0;
+  const int rot = 4 * ((tid >> 3) & 3) + ((tid & 7) >> 1);  // distinct banks across a warp
+#define ACS_CIDX(vt) (2 * (vt))
+#define ACS_RK(j) (seg0 + (((j) + rot) & (RAKE - 1)))
+#else
   const int seg0 = ((tid * RAKE) / VTHREADS) * LANE_STRIDE + v0 + (v0 >> 5);
+#define ACS_CIDX(vt) (2 * ((vt) + ((vt) >> 5)))
+#define ACS_RK(j) (seg0 + (j))
+#endif
   const int bb = pad32(tid * ITEMS);                        // my blocked items (contiguous)
   if (begin_bit >= end_bit) return;
 #pragma unroll
-  for (int j = 0; j < RAKE; ++j) s_cnt[seg0 + j] = 0u;
+  for (int j = 0; j < RAKE; ++j) s_cnt[ACS_RK(j)] = 0u;
   __syncthreads();
   for (int bit = begin_bit; bit < end_bit; bit += RADIX_BITS) {
     const int nb = min(RADIX_BITS, end_bit - bit);
@@ -156,7 +177,7 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
         const int i = v * IPV + q;
         const int vt = tid * VT + v;
         const uint32_t d = (uint32_t)(k[i] >> bit) & mask;
-        cidx[i] = (int)(d & (CNT_LANES - 1)) * (2 * LANE_STRIDE) + (int)(d >> (RADIX_BITS - 1)) + 2 * (vt + (vt >> 5));
+        cidx[i] = (int)(d & (CNT_LANES - 1)) * (2 * LANE_STRIDE) + (int)(d >> (RADIX_BITS - 1)) + ACS_CIDX(vt);
         pre[i] = c16[cidx[i]];
         c16[cidx[i]] = (uint16_t)(pre[i] + 1u);
       }
@@ -165,7 +186,7 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
     uint32_t seg[RAKE];
     uint32_t sum = 0;
 #pragma unroll
-    for (int j = 0; j < RAKE; ++j) { seg[j] = s_cnt[seg0 + j]; sum += seg[j]; }
+    for (int j = 0; j < RAKE; ++j) { seg[j] = s_cnt[ACS_RK(j)]; sum += seg[j]; }
     uint32_t inc = sum;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
@@ -185,8 +206,25 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
     wpre = __shfl_sync(0xffffffffu, lane == 0 ? 0u : wpre, w);
     // digits in the high halves follow all digits in the low halves
     uint32_t run = wpre + inc - sum + ((grand & 0xFFFFu) << 16);
+#if ACS_ROT_RAKE
+    {
+      // seg[m] holds counter (m + rot) mod 16 of the segment; its natural exclusive
+      // prefix is R(m) - H + (m < 16 - rot ? sum : 0), R the rotated running sum and
+      // H the sum of the first 16 - rot rotated words
+      uint32_t H = 0, R = 0;
+#pragma unroll
+      for (int j = 0; j < RAKE; ++j) H += j < RAKE - rot ? seg[j] : 0u;
+#pragma unroll
+      for (int j = 0; j < RAKE; ++j) {
+        // every packed half stays non-negative: no borrow between the two digits
+        s_cnt[ACS_RK(j)] = run + (j < RAKE - rot ? (sum - H) + R : R - H);
+        R += seg[j];
+      }
+    }
+#else
 #pragma unroll
     for (int j = 0; j < RAKE; ++j) { const uint32_t v = seg[j]; s_cnt[seg0 + j] = run; run += v; }
+#endif
     __syncthreads();
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) {
@@ -198,10 +236,12 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
     for (int i = 0; i < ITEMS; ++i) k[i] = s_words[bb + i];
     if (bit + RADIX_BITS < end_bit) {
 #pragma unroll
-      for (int j = 0; j < RAKE; ++j) s_cnt[seg0 + j] = 0u;
+      for (int j = 0; j < RAKE; ++j) s_cnt[ACS_RK(j)] = 0u;
       __syncthreads();
     }
   }
+#undef ACS_CIDX
+#undef ACS_RK
 }
 
 // =====================================================================
