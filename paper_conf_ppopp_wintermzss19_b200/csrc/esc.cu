@@ -248,18 +248,29 @@ __global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
     // ---------------- expand (L340) ----------------
     int col[ITEMS];
     int rmin = INT_MAX, rmax = INT_MIN, cmin = INT_MAX, cmax = INT_MIN;
+    // B addresses first, then all B loads of a half in flight, then the products
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-      if (ares[i] >= 0) {
-        const int e = ares[i];
-        const int q = S.a_bstart[e] + bres[i];
-        col[i] = __ldg(bcol + q);
-        S.s.vals[st.kept + i * THREADS + tid] = S.a_val[e] * __ldg(bval + q);
-        const int lr = S.a_lrow[e];
-        rmin = min(rmin, lr); rmax = max(rmax, lr);
-        cmin = min(cmin, col[i]); cmax = max(cmax, col[i]);
-      } else {
-        col[i] = 0;
+    for (int i = 0; i < ITEMS; ++i) bres[i] = ares[i] >= 0 ? S.a_bstart[ares[i]] + bres[i] : 0;
+    constexpr int HALF = ITEMS / 2;
+#pragma unroll
+    for (int h = 0; h < ITEMS; h += HALF) {
+      T bv[HALF];
+#pragma unroll
+      for (int u = 0; u < HALF; ++u) {
+        const int i = h + u;
+        if (ares[i] >= 0) { col[i] = __ldg(bcol + bres[i]); bv[u] = __ldg(bval + bres[i]); }
+        else { col[i] = 0; bv[u] = (T)0; }
+      }
+#pragma unroll
+      for (int u = 0; u < HALF; ++u) {
+        const int i = h + u;
+        if (ares[i] >= 0) {
+          const int e = ares[i];
+          S.s.vals[st.kept + i * THREADS + tid] = S.a_val[e] * bv[u];
+          const int lr = S.a_lrow[e];
+          rmin = min(rmin, lr); rmax = max(rmax, lr);
+          cmin = min(cmin, col[i]); cmax = max(cmax, col[i]);
+        }
       }
     }
 #pragma unroll
