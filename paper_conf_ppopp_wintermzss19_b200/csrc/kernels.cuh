@@ -77,7 +77,8 @@ struct MergeLists {
   int32_t* multi_idx;            // [nshared]
   int32_t* path_idx;
   int32_t* search_idx;
-  int64_t* counts_dev;           // [8]: nmulti, npath, nsearch, multi_total, merge_total, ngroups
+  int32_t* pair_idx;             // two-chunk rows of <= PAIR_MAX elements (warp merge)
+  int64_t* counts_dev;           // [8]: nmulti, npath, nsearch, npair, merge_total, -, multi_total
   int64_t* merge_total_scan;     // [nshared] exclusive scan of totals -> merge offsets
   int64_t* multi_scan;           // [nshared]
   int32_t* group_of;             // [nshared]
@@ -105,6 +106,7 @@ struct MergeArgs {
   int32_t* error_flag;
 };
 void launch_multi_merge(const MergeArgs& a, bool f64, cudaStream_t st);
+void launch_pair_merge(const MergeArgs& a, bool f64, cudaStream_t st);
 void launch_path_merge(const MergeArgs& a, bool f64, cudaStream_t st);
 void launch_search_merge(const MergeArgs& a, bool f64, cudaStream_t st);
 

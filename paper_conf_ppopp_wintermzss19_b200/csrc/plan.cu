@@ -66,7 +66,7 @@ struct acspgemm_plan_s {
   // buffers
   DevBuf seg, seg_rows, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base;
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
-  DevBuf kflag, kpos, lmulti, lpath, lsearch, mscan, mtscan, group_of, gstart, merge_col, merge_val;
+  DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan;
   int64_t* h_scal = nullptr;     // pinned read-back buffer
   cudaEvent_t ev[NSTAGE_EV];
@@ -140,7 +140,7 @@ int64_t helper_bytes(acspgemm_plan p) {
   DevBuf* bs[] = {&p->seg, &p->seg_rows, &p->scal, &p->brs, &p->nzb, &p->nze, &p->bprod, &p->bslot,
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->descs, &p->dense, &p->sflag,
                   &p->spos, &p->shared, &p->row_count, &p->row_ptr, &p->scan_tmp, &p->kflag, &p->kpos,
-                  &p->lmulti, &p->lpath, &p->lsearch, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
+                  &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
                   &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan};
   int64_t t = 0;
   for (DevBuf* b : bs) t += (int64_t)b->bytes;
@@ -324,13 +324,14 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   p->info.nshared = p->nshared;
   p->info.chunk_elems = p->h_scal[2];
   const int64_t nsh = p->nshared;
-  int64_t nmulti = 0, npath = 0, nsearch = 0, merge_total = 0, ngroups = 0;
+  int64_t nmulti = 0, npath = 0, nsearch = 0, npair = 0, merge_total = 0, ngroups = 0;
   if (nsh > 0) {
     ACS_ENSURE(p->kflag, sizeof(int32_t) * nsh);
     ACS_ENSURE(p->kpos, sizeof(int64_t) * nsh);
     ACS_ENSURE(p->lmulti, sizeof(int32_t) * nsh);
     ACS_ENSURE(p->lpath, sizeof(int32_t) * nsh);
     ACS_ENSURE(p->lsearch, sizeof(int32_t) * nsh);
+    ACS_ENSURE(p->lpair, sizeof(int32_t) * nsh);
     ACS_ENSURE(p->mtscan, sizeof(int64_t) * nsh);
     ACS_ENSURE(p->mscan, sizeof(int64_t) * nsh);
     ACS_ENSURE(p->group_of, sizeof(int32_t) * nsh);
@@ -342,6 +343,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     L.multi_idx = ptr<int32_t>(p->lmulti);
     L.path_idx = ptr<int32_t>(p->lpath);
     L.search_idx = ptr<int32_t>(p->lsearch);
+    L.pair_idx = ptr<int32_t>(p->lpair);
     L.counts_dev = scal + 8;
     L.merge_total_scan = ptr<int64_t>(p->mtscan);
     L.multi_scan = ptr<int64_t>(p->mscan);
@@ -349,12 +351,13 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     L.group_start = nullptr;
     L.scan_tmp = ptr<int64_t>(p->scan_tmp);
     launch_classify(L, st);
-    tl_launches += 3 * 5 + 1 + 3 + 1;
+    tl_launches += 4 * 5 + 1 + 3 + 1;
     ACS_CUDA(cudaGetLastError());
     if ((s = sync_read(p, scal + 8, 5, st)) != ACSPGEMM_OK) return s;
     nmulti = p->h_scal[0];
     npath = p->h_scal[1];
     nsearch = p->h_scal[2];
+    npair = p->h_scal[3];
     merge_total = p->h_scal[4];
     // Multi-Merge packing needs the multi totals: scan them over the multi list
     if (nmulti > 0) {
@@ -388,6 +391,9 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     ma.list = ptr<int32_t>(p->lmulti);
     ma.nlist = nmulti;
     if (nmulti > 0) { launch_multi_merge(ma, p->f64, st); tl_launches += 1; }
+    ma.list = ptr<int32_t>(p->lpair);
+    ma.nlist = npair;
+    if (npair > 0) { launch_pair_merge(ma, p->f64, st); tl_launches += 1; }
     record(p, S_PM, st);
     ma.list = ptr<int32_t>(p->lpath);
     ma.nlist = npath;
@@ -402,7 +408,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     record(p, S_PM, st);
     record(p, S_SM, st);
   }
-  p->info.nmulti = nmulti;
+  p->info.nmulti = nmulti + npair;
   p->info.npath = npath;
   p->info.nsearch = nsearch;
   p->info.nmulti_groups = ngroups;
@@ -587,7 +593,7 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
   DevBuf* bs[] = {&p->seg, &p->seg_rows, &p->scal, &p->brs, &p->nzb, &p->nze, &p->bprod, &p->bslot,
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->pool_col, &p->pool_val,
                   &p->descs, &p->dense, &p->sflag, &p->spos, &p->shared, &p->row_count, &p->row_ptr,
-                  &p->scan_tmp, &p->kflag, &p->kpos, &p->lmulti, &p->lpath, &p->lsearch, &p->mscan,
+                  &p->scan_tmp, &p->kflag, &p->kpos, &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan,
                   &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
                   &p->cur_last, &p->err, &p->bused, &p->bused_scan};
   for (DevBuf* b : bs) free_buf(*b);
