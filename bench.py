@@ -227,7 +227,24 @@ def main():
     stream = torch.cuda.current_stream()
 
     def step():
-        return plan.multiply(dA, dB, stream, A_view=view)
+        C = plan.multiply(dA, dB, stream, A_view=view)
+        if world > 1:
+            # the distributed C: per-rank pieces concatenated with row_ptr offsets, one
+            # all-gather of (rows, nnz) per rank
+            adist.gather_offsets(C.nnz, C.rows, device=dev)
+        return C
+
+    def digest(C, nnz_off):
+        # order-independent 64-bit sums of row_ptr (offset to the concatenated C, without
+        # the leading 0), column indices and value bits: equal for any GPU count
+        s_rp = int((C.row_ptr[1:].to(torch.int64) + nnz_off).sum().item())
+        s_col = int(C.col.to(torch.int64).sum().item())
+        vb = C.val.view(torch.int64) if C.val.dtype == torch.float64 else C.val.view(torch.int32).to(torch.int64)
+        s_val = int(vb.sum().item())
+        t = torch.tensor([s_rp, s_col, s_val], dtype=torch.int64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return "%016x-%016x-%016x" % tuple(int(x) & 0xFFFFFFFFFFFFFFFF for x in t.tolist())
 
     for _ in range(max(args.warmup, 0)):
         C = step()
@@ -269,6 +286,12 @@ def main():
     else:
         ms_step_max, products_all = ms_step, products
     value = 2.0 * products_all / (ms_step_max * 1e-3) / 1e9
+
+    # ---- determinism digest of C (untimed) ----
+    C = plan.multiply(dA, dB, stream, A_view=view)
+    off = adist.gather_offsets(C.nnz, C.rows, device=dev)[rank][1] if world > 1 else 0
+    c_digest = digest(C, off)
+    del C
 
     # ---- roofline of the dominant kernel (AC-ESC) ----
     esc_avg = sum(esc_ms) / len(esc_ms) if esc_ms else float("nan")
@@ -327,6 +350,7 @@ def main():
                                           "nsearch", "merge_elems", "pool_bytes", "helper_bytes",
                                           "pool_estimate_bytes")},
             "bcast_s": t_bcast,
+            "c_digest": c_digest,
         }
         print(json.dumps(out), flush=True)
     if world > 1:
