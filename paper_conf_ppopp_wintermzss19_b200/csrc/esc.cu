@@ -36,40 +36,18 @@ struct EscState {
   int64_t wofs;
 };
 
-// One local ESC iteration after expansion (values already at s.vals[pos]): build the
-// sort words, sort, compact (Alg. 3), emit completed rows as a chunk, keep the last row.
-template <typename Word, typename T>
-__device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, EscState& st, int consume,
-                                              int size_after, const int (&ares)[ITEMS], const int (&col)[ITEMS],
-                                              const int (&kc)[KEEP_PER_THREAD], int rmin, int cmin, int rowbits,
-                                              int colbits, int64_t pool_base, int64_t desc_base) {
+// Sort + compaction (Alg. 3) + emission of one local ESC iteration whose sort words are
+// already in s.words: completed rows become a chunk, the last row is kept.  Only the
+// key bits [IDXBITS, IDXBITS + sortbits) are sorted (0: words already sorted).
+// colof(key, pos) yields an element's output column.
+template <typename Word, typename T, typename ColOf>
+__device__ __forceinline__ void esc_tail(EscSmem<T>& S, const EscArgs& a, EscState& st, int n, int size_after,
+                                         int rmin, int sortbits, int colbits, int64_t pool_base, int64_t desc_base,
+                                         ColOf colof) {
   const int tid = threadIdx.x;
-  const int kept = st.kept;
-  const int n = kept + consume;
-  Word* sw = reinterpret_cast<Word*>(S.s.words);
-  // positions: kept elements first (they sort before equal keys, L366), then product c
-#pragma unroll
-  for (int i = 0; i < ITEMS; ++i) {
-    if (ares[i] >= 0) {
-      const int pos = kept + i * THREADS + tid;
-      const Word key = ((Word)(S.a_lrow[ares[i]] - rmin) << colbits) | (Word)(col[i] - cmin);
-      sw[pad32(pos)] = (key << IDXBITS) | (Word)pos;
-    }
-  }
-#pragma unroll
-  for (int j = 0; j < KEEP_PER_THREAD; ++j) {
-    const int p = j * THREADS + tid;
-    if (p < kept) {
-      const Word key = ((Word)(st.kept_lrow - rmin) << colbits) | (Word)(kc[j] - cmin);
-      sw[pad32(p)] = (key << IDXBITS) | (Word)p;
-    }
-  }
-  for (int p = n + tid; p < CAP; p += THREADS) sw[pad32(p)] = ~(Word)0;
-  __syncthreads();
-
   Word k[ITEMS];
   T ev[ITEMS];
-  load_and_sort<Word, T>(S.s, rowbits + colbits, k);
+  load_and_sort<Word, T>(S.s, sortbits, k);
   const ScanCtx<Word, T> ctx = compaction_prepare<Word, T>(S.s, k, n, colbits, ev);
   int* stage_col = reinterpret_cast<int*>(S.s.words);
   T* stage_val = S.s.vals;
@@ -93,12 +71,11 @@ __device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, E
   // chunk and merged later)
   const bool keep = size_after > 0 && rc_last <= KEEP;
   const int nchunk = total - (keep ? rc_last : 0);
-  const Word colmask = colbits ? (((Word)1 << colbits) - (Word)1) : (Word)0;
   // compacted element p goes to staging slot p: [0, nchunk) is the chunk, the kept
   // row stays at [nchunk, total) for the next iteration
   compaction_emit<Word, T>(k, ev, n, colbits, ctx, [&](int, Word key, T val, uint32_t state, bool row_end) {
     const int p = st_count(state) - 1;
-    stage_col[p] = cmin + (int)(key & colmask);
+    stage_col[p] = colof(key, 0);
     stage_val[p] = val;
     if (row_end && p < nchunk) {
       const int rc = st_row_count(state);
@@ -139,6 +116,106 @@ __device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, E
     st.kept_cmax = stage_col[total - 1];
   }
   __syncthreads();
+}
+
+
+// Radix path: key = (local row - rmin, column - cmin), all key bits sorted.
+// One local ESC iteration after expansion (values already at s.vals[pos]): build the
+// sort words, sort, compact (Alg. 3), emit completed rows as a chunk, keep the last row.
+template <typename Word, typename T>
+__device__ __forceinline__ void esc_iteration(EscSmem<T>& S, const EscArgs& a, EscState& st, int consume,
+                                              int size_after, const int (&ares)[ITEMS], const int (&col)[ITEMS],
+                                              const int (&kc)[KEEP_PER_THREAD], int rmin, int cmin, int rowbits,
+                                              int colbits, int64_t pool_base, int64_t desc_base) {
+  const int tid = threadIdx.x;
+  const int kept = st.kept;
+  const int n = kept + consume;
+  Word* sw = reinterpret_cast<Word*>(S.s.words);
+  // positions: kept elements first (they sort before equal keys, L366), then product c
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    if (ares[i] >= 0) {
+      const int pos = kept + i * THREADS + tid;
+      const Word key = ((Word)(S.a_lrow[ares[i]] - rmin) << colbits) | (Word)(col[i] - cmin);
+      sw[pad32(pos)] = (key << IDXBITS) | (Word)pos;
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < KEEP_PER_THREAD; ++j) {
+    const int p = j * THREADS + tid;
+    if (p < kept) {
+      const Word key = ((Word)(st.kept_lrow - rmin) << colbits) | (Word)(kc[j] - cmin);
+      sw[pad32(p)] = (key << IDXBITS) | (Word)p;
+    }
+  }
+  for (int p = n + tid; p < CAP; p += THREADS) sw[pad32(p)] = ~(Word)0;
+  __syncthreads();
+  const Word colmask = colbits ? (((Word)1 << colbits) - (Word)1) : (Word)0;
+  esc_tail<Word, T>(S, a, st, n, size_after, rmin, rowbits + colbits, colbits, pool_base, desc_base,
+                    [&](Word key, int) { return cmin + (int)(key & colmask); });
+}
+
+
+// Split-word path for keys of 21..31 bits (R-MAT, LP: 20-bit columns plus row bits):
+// instead of 64-bit sort words, sort 32-bit words (low 20 key bits | position) over
+// their key bits, then the remaining high key bits, read by position from a 16-bit side
+// array, in further stable passes.  Halves the shared-memory traffic of every pass.
+// The sorted words are then widened to 64-bit (key | position) for the compaction.
+template <typename T>
+__device__ __forceinline__ void esc_iteration_split(EscSmem<T>& S, const EscArgs& a, EscState& st, int consume,
+                                                    int size_after, const int (&ares)[ITEMS], const int (&col)[ITEMS],
+                                                    const int (&kc)[KEEP_PER_THREAD], int rmin, int cmin, int rowbits,
+                                                    int colbits, int64_t pool_base, int64_t desc_base) {
+  constexpr int LOBITS = 31 - IDXBITS;                      // 20: pads (all ones) stay last
+  const int tid = threadIdx.x;
+  const int kept = st.kept;
+  const int n = kept + consume;
+  const int keybits = rowbits + colbits;
+  uint32_t* sw = reinterpret_cast<uint32_t*>(S.s.words);
+  uint16_t* hi16 = reinterpret_cast<uint16_t*>(S.s.words + CAP_PAD / 2);   // upper half of the buffer
+  const uint64_t lomask = (1ull << LOBITS) - 1ull;
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    if (ares[i] >= 0) {
+      const int pos = kept + i * THREADS + tid;
+      const uint64_t key = ((uint64_t)(S.a_lrow[ares[i]] - rmin) << colbits) | (uint64_t)(col[i] - cmin);
+      sw[pad32(pos)] = ((uint32_t)(key & lomask) << IDXBITS) | (uint32_t)pos;
+      hi16[pos] = (uint16_t)(key >> LOBITS);
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < KEEP_PER_THREAD; ++j) {
+    const int p = j * THREADS + tid;
+    if (p < kept) {
+      const uint64_t key = ((uint64_t)(st.kept_lrow - rmin) << colbits) | (uint64_t)(kc[j] - cmin);
+      sw[pad32(p)] = ((uint32_t)(key & lomask) << IDXBITS) | (uint32_t)p;
+      hi16[p] = (uint16_t)(key >> LOBITS);
+    }
+  }
+  for (int p = n + tid; p < CAP; p += THREADS) { sw[pad32(p)] = ~0u; hi16[p] = 0xFFFFu; }
+  __syncthreads();
+  uint32_t k[ITEMS];
+  const int bb = pad32(tid * ITEMS);
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) k[i] = sw[bb + i];
+  block_radix_sort<uint32_t>(k, sw, S.s.u.cnt, S.s.swarp, IDXBITS, IDXBITS + LOBITS);
+  __syncthreads();
+  block_radix_sort<uint32_t>(k, sw, S.s.u.cnt, S.s.swarp, 0, keybits - LOBITS,
+                             [&](uint32_t w, int bit) { return (uint32_t)hi16[w & (uint32_t)(CAP - 1)] >> bit; });
+  uint64_t k64[ITEMS];
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) {
+    const uint32_t pos = k[i] & (uint32_t)(CAP - 1);
+    const uint64_t key = ((uint64_t)hi16[pos] << LOBITS) | (uint64_t)(k[i] >> IDXBITS);
+    k64[i] = tid * ITEMS + i < n ? ((key << IDXBITS) | pos) : ~0ull;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < ITEMS; ++i) S.s.words[bb + i] = k64[i];
+  __syncthreads();
+  const uint64_t colmask = colbits ? ((1ull << colbits) - 1ull) : 0ull;
+  esc_tail<uint64_t, T>(S, a, st, n, size_after, rmin, 0, colbits, pool_base, desc_base,
+                        [&](uint64_t key, int) { return cmin + (int)(key & colmask); });
 }
 
 template <typename T>
@@ -289,6 +366,9 @@ __global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
     if (rowbits + colbits + IDXBITS < 32)
       esc_iteration<uint32_t, T>(S, a, st, consume, size_after, ares, col, kc, rmin, cmin, rowbits, colbits,
                                  pool_base, desc_base);
+    else if (rowbits + colbits <= 31 - IDXBITS + 16)
+      esc_iteration_split<T>(S, a, st, consume, size_after, ares, col, kc, rmin, cmin, rowbits, colbits,
+                             pool_base, desc_base);
     else
       esc_iteration<uint64_t, T>(S, a, st, consume, size_after, ares, col, kc, rmin, cmin, rowbits, colbits,
                                  pool_base, desc_base);

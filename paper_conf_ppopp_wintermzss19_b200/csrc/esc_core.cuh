@@ -140,9 +140,16 @@ static_assert(VTHREADS % 32 == 0 && RAKE <= 32 && 32 % RAKE == 0, "raking layout
 static_assert(ITEMS <= 32 && 32 % ITEMS == 0, "blocked items must not straddle padding");
 static_assert(ITEMS % VT == 0, "virtual threads split the items evenly");
 
-template <typename Word>
+struct ShiftDigit {
+  template <typename Word>
+  __device__ __forceinline__ uint32_t operator()(Word w, int bit) const { return (uint32_t)(w >> bit); }
+};
+
+// digit(word, bit) >> 0 & mask is the digit of a pass (default: the word's own bits)
+template <typename Word, typename Digit = ShiftDigit>
 __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words, uint32_t* s_cnt,
-                                                 uint32_t* s_warp, int begin_bit, int end_bit) {
+                                                 uint32_t* s_warp, int begin_bit, int end_bit,
+                                                 Digit digit = Digit()) {
   constexpr int IPV = ITEMS / VT;                           // items per virtual thread
   const int tid = threadIdx.x, lane = lane_id(), w = warp_id();
   uint16_t* c16 = reinterpret_cast<uint16_t*>(s_cnt);
@@ -176,7 +183,7 @@ __device__ __forceinline__ void block_radix_sort(Word (&k)[ITEMS], Word* s_words
       for (int v = 0; v < VT; ++v) {
         const int i = v * IPV + q;
         const int vt = tid * VT + v;
-        const uint32_t d = (uint32_t)(k[i] >> bit) & mask;
+        const uint32_t d = digit(k[i], bit) & mask;
         cidx[i] = (int)(d & (CNT_LANES - 1)) * (2 * LANE_STRIDE) + (int)(d >> (RADIX_BITS - 1)) + ACS_CIDX(vt);
         pre[i] = c16[cidx[i]];
         c16[cidx[i]] = (uint16_t)(pre[i] + 1u);

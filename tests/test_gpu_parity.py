@@ -39,9 +39,9 @@ def gpu_mult(A, B, dt, plan=None, **kw):
     return C.to_numpy()
 
 
-def assert_parity(A, B, dt, exact=False, **kw):
+def assert_parity(A, B, dt, exact=False, oracle_threads=0, **kw):
     rp, col, val = gpu_mult(A, B, dt, **kw)
-    ref = oracle.gustavson(A.astype(dt), B.astype(dt))
+    ref = oracle.gustavson(A.astype(dt), B.astype(dt), threads=oracle_threads)
     assert rp.shape[0] == ref.row_ptr.shape[0]
     assert (rp == ref.row_ptr).all(), "row_ptr mismatch"
     assert (col == ref.col).all(), "col mismatch"
@@ -312,3 +312,36 @@ def test_sort_compact_vs_alg3(seed, cuda_available):
     assert [r[3] for r in ref] == ost.tolist()
     runend = (ost & 1).astype(bool)
     assert (oval[runend] == np.array([r[2] for r in ref])[runend]).all()
+
+
+@pytest.mark.parametrize("ncols_log2", [16, 24])
+def test_wide_column_ranges(ncols_log2, cuda_available):
+    """Column ranges that need 32-bit sort words (16) and the split 32-bit + side-array
+    words (24) in AC-ESC; B has few rows with columns spread over 2^ncols_log2.  (The
+    oracle's dense accumulator is as wide as C: one oracle thread keeps it small.)"""
+    rng = np.random.default_rng(ncols_log2)
+    K, ncols = 64, 1 << ncols_log2
+    A = random_rowlen_csr(600, K, rng.integers(1, 40, 600), seed=ncols_log2)
+    rows, cols = [], []
+    for r in range(K):
+        c = np.unique(rng.integers(0, ncols, int(rng.integers(1, 200))))
+        rows.append(np.full(c.size, r))
+        cols.append(c)
+    rows, cols = np.concatenate(rows), np.concatenate(cols)
+    B = from_coo(K, ncols, rows, cols, rng.uniform(-1, 1, rows.size))
+    assert_parity(A, B, np.float64, oracle_threads=1)
+    Bi = from_coo(K, ncols, rows, cols, rng.integers(-3, 4, rows.size).astype(np.float64))
+    Ai = random_rowlen_csr(600, K, rng.integers(1, 40, 600), seed=ncols_log2 + 1, values="int")
+    assert_parity(Ai, Bi, np.float64, exact=True, oracle_threads=1)
+
+
+def test_64bit_sort_words(cuda_available):
+    """Keys wider than the split path (> 36 bits): 512 one-entry rows per block (9 row
+    bits) times columns spread over 2^28 -> 64-bit sort words."""
+    rng = np.random.default_rng(5)
+    K, ncols = 32, 1 << 28
+    A = from_coo(4096, K, np.arange(4096), rng.integers(0, K, 4096), rng.integers(1, 4, 4096).astype(np.float64))
+    rows = np.repeat(np.arange(K), 4)
+    cols = np.concatenate([np.sort(rng.choice(ncols, 4, replace=False)) for _ in range(K)])
+    B = from_coo(K, ncols, rows, cols, rng.integers(-3, 4, rows.size).astype(np.float64))
+    assert_parity(A, B, np.float64, exact=True, oracle_threads=1)
