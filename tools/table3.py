@@ -1,0 +1,46 @@
+"""Table-3-style memory report (Table 3) for the synthetic workloads:
+helper memory, chunk pool reserved (exact per-block bound, reading R8) next to the
+paper's pool estimate (L556), chunk memory used, used/output (u/o), restarts (always 0:
+the deterministic allocator never restarts) and nnz(C).  Run on a GPU box:
+    python tools/table3.py > profiles/r1_table3.md
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import paper_conf_ppopp_wintermzss19_b200 as acs  # noqa: E402
+from synth import aggregation_prolongator, config, poisson3d_7pt  # noqa: E402
+
+
+def row(name, A, B, dt):
+    vb = np.dtype(dt).itemsize
+    dA = acs.DeviceCSR.from_host(A, "cuda", dt)
+    dB = dA if B is A else acs.DeviceCSR.from_host(B, "cuda", dt)
+    plan = acs.Plan()
+    C = plan.multiply(dA, dB)
+    torch.cuda.synchronize()
+    i = plan.info()
+    used = i["chunk_elems"] * (4 + vb)
+    out = i["nnz_c"] * (4 + vb)
+    MB = 1e6
+    line = (f"| {name} | {np.dtype(dt).name} | {i['helper_bytes'] / MB:.1f} | {i['pool_bytes'] / MB:.1f} | "
+            f"{i['pool_estimate_bytes'] / MB:.1f} | {used / MB:.1f} | {100 * used / max(i['pool_bytes'], 1):.1f} % | "
+            f"{used / max(out, 1):.2f} | 0 | {i['nnz_c']:,} | {i['nchunks']:,} | {i['nshared']:,} |")
+    print(line, flush=True)
+    del C, dA, dB
+    plan.close()
+    torch.cuda.empty_cache()
+
+
+print("| workload | dtype | helper MB | pool MB (exact bound) | pool MB (paper estimate) | used MB | % | u/o | restarts | nnz(C) | chunks | shared rows |")
+print("|---|---|---|---|---|---|---|---|---|---|---|---|")
+for cfg in ("cfg1", "cfg2", "cfg3", "cfg5"):
+    A, B = config(cfg)
+    row(cfg, A, B if cfg == "cfg5" else A, np.float64)
+A = poisson3d_7pt(256)
+row("cfg4a A·P", A, aggregation_prolongator(256), np.float64)
