@@ -141,7 +141,15 @@ acspgemm_status acspgemm_numeric(acspgemm_plan plan, acspgemm_csr_out* C, void* 
 acspgemm_status acspgemm_multiply(const acspgemm_csr_in* A, const acspgemm_csr_in* B, acspgemm_csr_out* C,
                                   void* stream, acspgemm_dtype dtype);
 
-/* Free C allocated by acspgemm_multiply (cudaFreeAsync on `stream`). */
+/* Galerkin triple product C = R·(A·P) as two ordered AC-SpGEMMs (SURVEY §8(f)-2,
+ * reading R24: the association R·(A·P)).  A·P lives in temporary device memory that is
+ * released before return; C is allocated like acspgemm_multiply (cudaMallocAsync on
+ * `stream`, free with acspgemm_free_csr).  Requires R.cols == A.rows, A.cols == P.rows.
+ * Synchronises `stream`. */
+acspgemm_status acspgemm_rap(const acspgemm_csr_in* R, const acspgemm_csr_in* A, const acspgemm_csr_in* P,
+                             acspgemm_csr_out* C, void* stream, acspgemm_dtype dtype);
+
+/* Free C allocated by acspgemm_multiply or acspgemm_rap (cudaFreeAsync on `stream`). */
 acspgemm_status acspgemm_free_csr(acspgemm_csr_out* C, void* stream);
 
 /* Per-stage device times (ms) of the last symbolic + numeric when collect_stage_times

@@ -176,6 +176,40 @@ def multiply(A: DeviceCSR, B: DeviceCSR, stream=None, **plan_kw) -> DeviceCSR:
         p.close()
 
 
+def rap(R: DeviceCSR, A: DeviceCSR, P: DeviceCSR, stream=None, **plan_kw) -> DeviceCSR:
+    """Galerkin triple product R·(A·P) (two ordered multiplies, C allocated by torch)."""
+    if R.cols != A.rows or A.cols != P.rows:
+        raise ValueError("dimension mismatch")
+    p = Plan(**plan_kw)
+    try:
+        AP = p.multiply(A, P, stream)
+        return p.multiply(R, AP, stream)
+    finally:
+        p.close()
+
+
+def rap_lib_alloc(R: DeviceCSR, A: DeviceCSR, P: DeviceCSR, stream=None):
+    """R·(A·P) through acspgemm_rap (library-allocated C); returns host numpy arrays."""
+    lib = load()
+    r, a_, p_ = _csr_in(R), _csr_in(A), _csr_in(P)
+    c = CsrOut()
+    st = _stream_ptr(stream)
+    check(lib.acspgemm_rap(ctypes.byref(r), ctypes.byref(a_), ctypes.byref(p_), ctypes.byref(c), st,
+                           _dtype_code(A.dtype)), "acspgemm_rap")
+    try:
+        rp = np.empty(c.rows + 1, dtype=np.int32)
+        col = np.empty(c.nnz, dtype=np.int32)
+        val = np.empty(c.nnz, dtype=np.float64 if A.dtype == torch.float64 else np.float32)
+        torch.cuda.synchronize()
+        _memcpy_d2h(rp, c.row_ptr)
+        _memcpy_d2h(col, c.col_idx)
+        _memcpy_d2h(val, c.val)
+        return rp, col, val
+    finally:
+        check(lib.acspgemm_free_csr(ctypes.byref(c), st), "acspgemm_free_csr")
+        torch.cuda.synchronize()
+
+
 def multiply_lib_alloc(A: DeviceCSR, B: DeviceCSR, stream=None):
     """C = A·B through acspgemm_multiply (the library allocates C with cudaMallocAsync).
     Returns host numpy arrays (row_ptr, col, val) and frees the device C."""

@@ -673,6 +673,20 @@ acspgemm_status acspgemm_multiply(const acspgemm_csr_in* A, const acspgemm_csr_i
   return s;
 }
 
+acspgemm_status acspgemm_rap(const acspgemm_csr_in* R, const acspgemm_csr_in* A, const acspgemm_csr_in* P,
+                             acspgemm_csr_out* C, void* stream, acspgemm_dtype dtype) {
+  if (!R || !A || !P || !C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
+  if (R->cols != A->rows) return set_err(ACSPGEMM_ERR_DIM_MISMATCH, "R.cols != A.rows");
+  acspgemm_csr_out AP{};
+  acspgemm_status s = acspgemm_multiply(A, P, &AP, stream, dtype);
+  if (s != ACSPGEMM_OK) return s;
+  const acspgemm_csr_in APin{AP.rows, AP.cols, AP.nnz, AP.row_ptr, AP.col_idx, AP.val};
+  s = acspgemm_multiply(R, &APin, C, stream, dtype);
+  acspgemm_free_csr(&AP, stream);
+  if (s == ACSPGEMM_OK) ACS_CUDA(cudaStreamSynchronize(reinterpret_cast<cudaStream_t>(stream)));
+  return s;
+}
+
 acspgemm_status acspgemm_free_csr(acspgemm_csr_out* C, void* stream) {
   if (!C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C is NULL");
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);

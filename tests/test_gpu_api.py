@@ -176,3 +176,18 @@ def test_fp32_bit_identical_across_segment_splits(cuda_available):
     from paper_conf_ppopp_wintermzss19_b200.dist import concat_pieces
     rp, col, val = concat_pieces(pieces)
     assert (rp == frp).all() and (col == fcol).all() and val.tobytes() == fval.tobytes()
+
+
+def test_rap_galerkin(cuda_available):
+    """acspgemm_rap / rap: R·(A·P) = 4·A₇(n/2) exactly for 2³ aggregation (§8(f)-2)."""
+    from synth import aggregation_prolongator, poisson3d_7pt, transpose
+    p = pkg()
+    n = 16
+    A, P = poisson3d_7pt(n), aggregation_prolongator(n)
+    R = transpose(P)
+    A4 = poisson3d_7pt(n // 2)
+    C = p.rap(dev(R), dev(A), dev(P))
+    rp, col, val = C.to_numpy()
+    assert (rp == A4.row_ptr).all() and (col == A4.col).all() and (val == 4 * A4.val).all()
+    rp, col, val = p.rap_lib_alloc(dev(R), dev(A), dev(P))
+    assert (rp == A4.row_ptr).all() and (col == A4.col).all() and (val == 4 * A4.val).all()
