@@ -19,10 +19,12 @@ def run(name, A, B, dt, reps=5):
            "nshared": info["nshared"], "nmulti": info["nmulti"], "npath": info["npath"], "nsearch": info["nsearch"]}
     print(json.dumps(out), flush=True)
     plan.close(); del dA, dB; torch.cuda.empty_cache()
-for cfg in ["cfg1", "cfg2", "cfg3", "cfg5"]:
+CFGS = sys.argv[1].split(",") if len(sys.argv) > 1 else ["cfg1", "cfg2", "cfg3", "cfg5", "cfg4"]
+for cfg in [c for c in CFGS if c != "cfg4"]:
     for dt in ([np.float64, np.float32] if cfg != "cfg1" else [np.float64]):
         A, B = config(cfg, dt)
         run(cfg, A, B if cfg == "cfg5" else A, dt)
+if "cfg4" not in CFGS: sys.exit(0)
 A = poisson3d_7pt(256); P = aggregation_prolongator(256)
 run("cfg4a A*P", A, P, np.float64)
 import oracle

@@ -122,6 +122,43 @@ def test_long_rows_multi_chunk(seed, cuda_available):
     assert info["npath"] + info["nsearch"] > 0
 
 
+@pytest.mark.parametrize("ncols_log2", [11, 12, 13])
+def test_path_merge_windows_dense_columns(ncols_log2, cuda_available):
+    """Path Merge windows over rows that fill a power-of-two column range: the window's
+    largest key reaches 2^k - 1, padding words sit between the pieces' entries, and the
+    proportional staging cut (reading R12) must still rank them last."""
+    n = 1 << ncols_log2
+    rows, k = 8, 1500
+    rng = np.random.default_rng(ncols_log2)
+    r = np.repeat(np.arange(rows), k)
+    c = np.concatenate([np.sort(rng.choice(6000, k, replace=False)) for _ in range(rows)])
+    A = from_coo(rows, 6000, r, c, rng.uniform(-1, 1, rows * k))
+    B = random_rowlen_csr(6000, n, np.full(6000, 20), seed=ncols_log2, values="uniform")
+    plan = pkg().Plan()
+    assert_parity(A, B, np.float64, plan=plan)
+    assert plan.info()["npath"] >= 1
+
+
+def test_path_merge_window_all_ones_key(cuda_available):
+    """Deterministic Path Merge window whose largest key is all ones in its bit width.
+    A = one row (1, 1, 1); B rows of exactly CAP entries, so each ESC iteration emits one
+    B row as one chunk of C's row 0 (three pieces).  Proportional staging takes 682
+    entries per piece; piece 1's next column 1024 is the cut and lo = 0, so the window's
+    largest key is 1023 = 2^10 - 1 (piece 2) while piece 0's staged entries >= 1024 are
+    padding words in front of it: the sorted bits must rank the padding after 1023."""
+    rows = [list(range(0, 600)) + list(range(2000, 3448)),
+            list(range(0, 682)) + list(range(1024, 2390)),
+            list(range(300, 981)) + [1023] + list(range(3000, 4366))]
+    assert all(len(r) == 2048 for r in rows)
+    rng = np.random.default_rng(5)
+    B = from_coo(3, 5000, np.repeat(np.arange(3), 2048), np.concatenate(rows), rng.uniform(-1, 1, 3 * 2048))
+    A = from_coo(1, 3, [0, 0, 0], [0, 1, 2], np.array([1.0, -2.0, 0.5]))
+    plan = pkg().Plan()
+    assert_parity(A, B, np.float64, plan=plan)
+    info = plan.info()
+    assert info["npath"] == 1 and info["nchunks"] == 3
+
+
 def test_dense_row_search_merge(cuda_available):
     """One very long output row (> PATH_MAX_CHUNKS chunks) forces Search Merge."""
     n = 60000
