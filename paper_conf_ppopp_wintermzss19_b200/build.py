@@ -18,7 +18,7 @@ SOURCES = ["glb.cu", "scan.cu", "esc.cu", "merge.cu", "copy.cu", "plan.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr", "-ftz=false", "-prec-div=true",
-         "-prec-sqrt=true", "-fmad=true"]
+         "-prec-sqrt=true", "-fmad=true"] + os.environ.get("ACS_EXTRA_NVCC_FLAGS", "").split()
 
 
 def _stale(obj: str, deps) -> bool:
