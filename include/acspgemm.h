@@ -141,6 +141,23 @@ acspgemm_status acspgemm_numeric(acspgemm_plan plan, acspgemm_csr_out* C, void* 
 acspgemm_status acspgemm_multiply(const acspgemm_csr_in* A, const acspgemm_csr_in* B, acspgemm_csr_out* C,
                                   void* stream, acspgemm_dtype dtype);
 
+/* End-to-end C = A·B with A, B and C in HOST memory: inputs host -> device on `stream`,
+ * the multiply, the result device -> host.  A_host / B_host carry host pointers (page-
+ * locked memory gives asynchronous full-speed copies; pageable memory works, slower);
+ * B_host may alias A_host (copied once).  The multiply runs in `npieces` row pieces of
+ * whole canonical segments (1 <= npieces <= the plan's num_segments), so
+ * the device -> host copy of piece g (on an internal stream) overlaps the multiply of
+ * piece g + 1; C is bit-identical to a one-piece multiply.  C->row_ptr (rows+1 entries),
+ * C->col_idx and C->val (`capacity` entries) are caller-allocated HOST buffers.  If
+ * nnz(C) > capacity the call returns ACSPGEMM_ERR_INVALID_ARG with C->nnz = nnz(C), which
+ * makes capacity = 0 a size query.  The device copies of A and B and two alternating
+ * piece buffers of C are plan memory (kept for reuse until acspgemm_plan_destroy); the
+ * plan's segment setting is restored.  The plan's counters and stage times describe the
+ * last piece.  Synchronises `stream`. */
+acspgemm_status acspgemm_multiply_host(acspgemm_plan plan, const acspgemm_csr_in* A_host,
+                                       const acspgemm_csr_in* B_host, acspgemm_dtype dtype, void* stream,
+                                       int npieces, acspgemm_csr_out* C_host, int64_t capacity);
+
 /* Galerkin triple product C = R·(A·P) as two ordered AC-SpGEMMs (SURVEY §8(f)-2,
  * reading R24: the association R·(A·P)).  A·P lives in temporary device memory that is
  * released before return; C is allocated like acspgemm_multiply (cudaMallocAsync on

@@ -51,6 +51,8 @@ SIGNATURES = {
     "acspgemm_numeric": (ctypes.c_int, [VP, ctypes.POINTER(CsrOut), VP]),
     "acspgemm_multiply": (ctypes.c_int, [ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.POINTER(CsrOut), VP,
                                          ctypes.c_int]),
+    "acspgemm_multiply_host": (ctypes.c_int, [VP, ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.c_int, VP,
+                                              ctypes.c_int, ctypes.POINTER(CsrOut), I64]),
     "acspgemm_rap": (ctypes.c_int, [ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn),
                                     ctypes.POINTER(CsrOut), VP, ctypes.c_int]),
     "acspgemm_free_csr": (ctypes.c_int, [ctypes.POINTER(CsrOut), VP]),

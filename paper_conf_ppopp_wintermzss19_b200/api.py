@@ -147,6 +147,43 @@ class Plan:
         self.numeric(rp, col, val, stream)
         return DeviceCSR(rows, B.cols, rp, col[:nnz], val[:nnz])
 
+    def multiply_host(self, A, B, out=None, pieces: int = 4, stream=None):
+        """End to end through acspgemm_multiply_host: A and B on the host (objects with
+        rows, cols, row_ptr, col, val as numpy arrays or CPU tensors; int32 indices),
+        C returned on the host.  `out` = (row_ptr, col, val) host buffers (pinned CPU
+        tensors or numpy arrays; col/val capacity = their length); without it a size
+        query runs first and pinned tensors are allocated.  Returns (row_ptr, col, val)
+        trimmed to nnz(C)."""
+        dt = _host_dtype(A.val)
+        if _host_dtype(B.val) != dt:
+            raise TypeError("A and B must have the same value dtype")
+        a, keep_a = _host_csr_in(A)
+        b, keep_b = (a, keep_a) if B is A else _host_csr_in(B)
+        st = _stream_ptr(stream)
+        code = 1 if dt == np.float64 else 0
+        c = CsrOut()
+        if out is None:
+            rp = torch.empty(A.rows + 1, dtype=torch.int32).pin_memory()
+            c.row_ptr = rp.data_ptr()
+            st_code = self._lib.acspgemm_multiply_host(self._h, ctypes.byref(a), ctypes.byref(b), code, st,
+                                                       int(pieces), ctypes.byref(c), 0)
+            if st_code not in (0, 1):
+                check(st_code, "acspgemm_multiply_host")
+            n = int(c.nnz)
+            tdt = torch.float64 if dt == np.float64 else torch.float32
+            out = (rp, torch.empty(max(n, 1), dtype=torch.int32).pin_memory(),
+                   torch.empty(max(n, 1), dtype=tdt).pin_memory())
+        orp, ocol, oval = out
+        if len(orp) < A.rows + 1 or len(ocol) != len(oval):
+            raise ValueError("out buffers: row_ptr needs rows+1 entries, col and val the same capacity")
+        c = CsrOut()
+        c.row_ptr, c.col_idx, c.val = _host_ptr(orp), _host_ptr(ocol), _host_ptr(oval)
+        check(self._lib.acspgemm_multiply_host(self._h, ctypes.byref(a), ctypes.byref(b), code, st, int(pieces),
+                                               ctypes.byref(c), len(ocol)), "acspgemm_multiply_host")
+        n = int(c.nnz)
+        del keep_a, keep_b
+        return orp[:A.rows + 1], ocol[:n], oval[:n]
+
     def info(self) -> dict:
         inf = Info()
         check(self._lib.acspgemm_plan_info(self._h, ctypes.byref(inf)), "acspgemm_plan_info")
@@ -165,6 +202,48 @@ class Plan:
         check(self._lib.acspgemm_block_row_starts(self._h, out.ctypes.data_as(_lib.PI32), n),
               "acspgemm_block_row_starts")
         return out[:n]
+
+
+def _host_dtype(v):
+    if isinstance(v, torch.Tensor):
+        return {torch.float64: np.float64, torch.float32: np.float32}[v.dtype]
+    return np.dtype(v.dtype).type
+
+
+def _host_ptr(x) -> int:
+    if isinstance(x, torch.Tensor):
+        if x.is_cuda or not x.is_contiguous():
+            raise ValueError("host buffers must be contiguous CPU tensors")
+        return x.data_ptr()
+    if not x.flags["C_CONTIGUOUS"]:
+        raise ValueError("host arrays must be C-contiguous")
+    return x.ctypes.data
+
+
+def _host_csr_in(M):
+    """CsrIn over host arrays (int32 indices required; numpy arrays of another integer
+    type are converted, the returned list keeps the converted arrays alive)."""
+    keep = []
+    arrs = []
+    for x, want in ((M.row_ptr, np.int32), (M.col, np.int32), (M.val, None)):
+        if isinstance(x, torch.Tensor):
+            if want is not None and x.dtype != torch.int32:
+                raise TypeError("row_ptr / col must be int32")
+        elif want is not None and x.dtype != want:
+            x = np.ascontiguousarray(x, dtype=want)
+        keep.append(x)
+        arrs.append(_host_ptr(x))
+    nnz = int(M.row_ptr[M.rows]) - int(M.row_ptr[0]) if M.rows > 0 else 0
+    return CsrIn(M.rows, M.cols, nnz, arrs[0], arrs[1], arrs[2]), keep
+
+
+def multiply_host(A, B, out=None, pieces: int = 4, stream=None, **plan_kw):
+    """C = A·B with host inputs and host result (one-shot plan; see Plan.multiply_host)."""
+    p = Plan(**plan_kw)
+    try:
+        return p.multiply_host(A, B, out, pieces, stream)
+    finally:
+        p.close()
 
 
 def multiply(A: DeviceCSR, B: DeviceCSR, stream=None, **plan_kw) -> DeviceCSR:

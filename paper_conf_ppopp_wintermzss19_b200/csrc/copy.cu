@@ -7,6 +7,7 @@
 // a single contiguous copy.  Shared rows copy their merged data from the merge pool.
 // B200: one warp per chunk (chunks average a few hundred elements), streaming
 // (evict-first) loads and stores since neither side is re-read.
+#include <algorithm>
 #include "kernels.cuh"
 
 namespace acs {
@@ -60,6 +61,41 @@ void launch_copy(const CopyArgs& a, bool f64, cudaStream_t st) {
   const unsigned grid = (unsigned)((items + COPY_WARPS - 1) / COPY_WARPS);
   if (f64) k_copy<double><<<grid, 32 * COPY_WARPS, 0, st>>>(a);
   else k_copy<float><<<grid, 32 * COPY_WARPS, 0, st>>>(a);
+}
+
+// Small read-backs go to mapped host memory through the SM (a copy-engine transfer would
+// queue behind a large device->host copy running on another stream).
+__global__ void k_read_back(const uint32_t* __restrict__ src, volatile uint32_t* dst, int nwords) {
+  const int i = threadIdx.x;
+  if (i < nwords) dst[i] = src[i];
+}
+
+void launch_read_back(const void* src, void* mapped_dst, int nbytes, cudaStream_t st) {
+  const int nw = (nbytes + 3) / 4;
+  k_read_back<<<1, 32 * ((nw + 31) / 32), 0, st>>>(static_cast<const uint32_t*>(src),
+                                                   static_cast<uint32_t*>(mapped_dst), nw);
+}
+
+__global__ void k_copy_offset(int32_t* __restrict__ dst, const int32_t* __restrict__ src, int64_t n, int32_t off) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = src[i] + off;
+}
+
+void launch_copy_offset(int32_t* dst, const int32_t* src, int64_t n, int32_t off, cudaStream_t st) {
+  if (n <= 0) return;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 148 * 8);
+  k_copy_offset<<<grid, 256, 0, st>>>(dst, src, n, off);
+}
+
+__global__ void k_add_offset(int32_t* __restrict__ p, int64_t n, int32_t off) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] += off;
+}
+
+void launch_add_offset(int32_t* p, int64_t n, int32_t off, cudaStream_t st) {
+  if (n <= 0 || off == 0) return;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 148 * 8);
+  k_add_offset<<<grid, 256, 0, st>>>(p, n, off);
 }
 
 }  // namespace acs

@@ -126,6 +126,12 @@ struct CopyArgs {
   void* c_val;
 };
 void launch_copy(const CopyArgs& a, bool f64, cudaStream_t st);
+// dst[i] = src[i] + off (row pointers of a row piece placed after earlier pieces)
+void launch_copy_offset(int32_t* dst, const int32_t* src, int64_t n, int32_t off, cudaStream_t st);
+// nbytes (multiple of 4, <= 4096) from device memory to mapped host memory, by a kernel
+void launch_read_back(const void* src, void* mapped_dst, int nbytes, cudaStream_t st);
+// p[i] += off for i < n (row pointers of a row piece placed after earlier pieces)
+void launch_add_offset(int32_t* p, int64_t n, int32_t off, cudaStream_t st);
 
 // ---- validation ----------------------------------------------------------------
 void launch_validate(const CsrView& M, int32_t* bad_flag, cudaStream_t st);

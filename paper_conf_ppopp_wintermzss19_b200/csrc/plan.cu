@@ -55,6 +55,11 @@ struct DevBuf {
   size_t bytes = 0;
 };
 
+// mapped host buffer h_scal: [0, 32) read-backs, [32, 97) explicit segment rows (read by
+// the segments kernel), [97, 162) segment boundaries read back for acspgemm_info
+constexpr int H_SEG_ROWS = 32;
+constexpr int H_SEG_INFO = H_SEG_ROWS + MAX_SEGMENTS + 1;
+constexpr int H_SCAL_WORDS = H_SEG_INFO + MAX_SEGMENTS + 1;
 enum Stage { S_GLB = 0, S_ESC, S_MCC, S_MM, S_PM, S_SM, S_SCAN, S_CC, S_END, NSTAGE_EV };
 
 }  // namespace
@@ -68,6 +73,10 @@ struct acspgemm_plan_s {
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan;
+  // acspgemm_multiply_host: device copies of A and B, two C piece buffers, copy stream
+  DevBuf hp_a[3], hp_b[3], hp_c[2][3];
+  cudaStream_t hp_cs = nullptr;
+  cudaEvent_t hp_ready = nullptr, hp_copied[2] = {nullptr, nullptr};
   int64_t* h_scal = nullptr;     // pinned read-back buffer
   cudaEvent_t ev[NSTAGE_EV];
   bool ev_ok = false;
@@ -148,7 +157,8 @@ int64_t helper_bytes(acspgemm_plan p) {
 }
 
 acspgemm_status sync_read(acspgemm_plan p, const int64_t* dev, int n, cudaStream_t st) {
-  ACS_CUDA(cudaMemcpyAsync(p->h_scal, dev, sizeof(int64_t) * n, cudaMemcpyDeviceToHost, st));
+  launch_read_back(dev, p->h_scal, (int)sizeof(int64_t) * n, st);
+  tl_launches += 1;
   ACS_CUDA(cudaStreamSynchronize(st));
   return ACSPGEMM_OK;
 }
@@ -196,9 +206,10 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     launch_validate(Av, ptr<int32_t>(p->err), st);
     launch_validate(Bv, ptr<int32_t>(p->err), st);
     tl_launches += 2;
-    ACS_CUDA(cudaMemcpyAsync(p->h_scal, p->err.p, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+    launch_read_back(p->err.p, p->h_scal, sizeof(int32_t), st);
+    tl_launches += 1;
     ACS_CUDA(cudaStreamSynchronize(st));
-    if (*reinterpret_cast<int32_t*>(p->h_scal) != 0)
+    if (*reinterpret_cast<volatile int32_t*>(p->h_scal) != 0)
       return set_err(ACSPGEMM_ERR_INVALID_ARG, "input is not canonical CSR (row_ptr/col order/range)");
   }
 
@@ -214,9 +225,11 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   if (p->nseg_explicit > 0) {
     if (p->seg_rows_explicit[p->nseg_explicit] != A->rows)
       return set_err(ACSPGEMM_ERR_INVALID_ARG, "explicit segments do not end at A.rows");
-    ACS_CUDA(cudaMemcpyAsync(p->seg_rows.p, p->seg_rows_explicit, sizeof(int64_t) * (nseg + 1),
-                             cudaMemcpyHostToDevice, st));
-    explicit_rows = ptr<int64_t>(p->seg_rows);
+    // through mapped host memory (no copy engine: see launch_read_back); the previous
+    // symbolic has synchronised, so no kernel still reads the old values
+    int64_t* hs = p->h_scal + H_SEG_ROWS;
+    for (int i = 0; i <= nseg; ++i) hs[i] = p->seg_rows_explicit[i];
+    explicit_rows = hs;
   }
   ACS_ENSURE(p->brs, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->nzb, sizeof(int32_t) * max_blocks);
@@ -245,17 +258,15 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   k_put_i64<<<1, 1, 0, st>>>(scal + 2, nblocks_dev);
   tl_launches += 1;
   ACS_CUDA(cudaGetLastError());
+  // segment boundaries (for info) ride along with the first read-back
+  launch_read_back(p->seg.p, p->h_scal + H_SEG_INFO, (int)sizeof(int64_t) * (nseg + 1), st);
+  tl_launches += 1;
   if ((s = sync_read(p, scal, 3, st)) != ACSPGEMM_OK) return s;
   const int64_t products = p->h_scal[0], slots = p->h_scal[1], nblocks = p->h_scal[2];
   p->info.products = products;
   p->info.nblocks = nblocks;
   p->info.nsegments = nseg;
-  {
-    // segment boundaries for info (tiny copy)
-    int64_t segtab[MAX_SEGMENTS + 1];
-    ACS_CUDA(cudaMemcpy(segtab, p->seg.p, sizeof(int64_t) * (nseg + 1), cudaMemcpyDeviceToHost));
-    for (int i = 0; i <= nseg; ++i) p->info.segment_rows[i] = segtab[i];
-  }
+  for (int i = 0; i <= nseg; ++i) p->info.segment_rows[i] = p->h_scal[H_SEG_INFO + i];
   const int64_t pool_bytes = products * (4 + vbytes);
   if (p->opt.pool_limit_bytes && (size_t)pool_bytes > p->opt.pool_limit_bytes)
     return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, "exact chunk-pool bound " + std::to_string(pool_bytes) +
@@ -421,8 +432,9 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
                      ptr<int64_t>(p->scan_tmp), st);
   tl_launches += 3;
   ACS_CUDA(cudaGetLastError());
-  ACS_CUDA(cudaMemcpyAsync(p->h_scal, scal + 16, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
-  ACS_CUDA(cudaMemcpyAsync(p->h_scal + 1, p->err.p, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  launch_read_back(scal + 16, p->h_scal, sizeof(int64_t), st);
+  launch_read_back(p->err.p, p->h_scal + 1, sizeof(int32_t), st);
+  tl_launches += 2;
   record(p, S_CC, st);
   ACS_CUDA(cudaStreamSynchronize(st));
   const int64_t nnz = p->h_scal[0];
@@ -438,7 +450,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   return ACSPGEMM_OK;
 }
 
-acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t st) {
+acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t st, int32_t row_off = 0) {
   if (!p->ready) return set_err(ACSPGEMM_ERR_NOT_READY, "numeric called without a successful symbolic");
   if (!C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C is NULL");
   if (p->rows > 0 && !C->row_ptr) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C.row_ptr is NULL");
@@ -448,11 +460,15 @@ acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t 
   C->cols = p->cols;
   C->nnz = p->nnz;
   if (p->empty) {
-    if (p->rows >= 0 && C->row_ptr) ACS_CUDA(cudaMemsetAsync(C->row_ptr, 0, sizeof(int32_t) * (p->rows + 1), st));
+    if (p->rows >= 0 && C->row_ptr) {
+      ACS_CUDA(cudaMemsetAsync(C->row_ptr, 0, sizeof(int32_t) * (p->rows + 1), st));
+      launch_add_offset(C->row_ptr, p->rows + 1, row_off, st);
+    }
     p->info.kernel_launches = p->launches_sym;
     return ACSPGEMM_OK;
   }
-  ACS_CUDA(cudaMemcpyAsync(C->row_ptr, p->row_ptr.p, sizeof(int32_t) * (p->rows + 1), cudaMemcpyDeviceToDevice, st));
+  launch_copy_offset(C->row_ptr, ptr<int32_t>(p->row_ptr), p->rows + 1, row_off, st);
+  tl_launches += 1;
   record(p, S_CC, st);
   CopyArgs ca;
   ca.dense = ptr<ChunkDesc>(p->dense);
@@ -543,6 +559,24 @@ __global__ void k_debug_sort_compact(const int32_t* rows, const int32_t* cols, c
   });
 }
 
+// Restores a plan's explicit segments when acspgemm_multiply_host returns (any path)
+// and leaves both of its streams idle.
+struct HostPipeGuard {
+  acspgemm_plan plan;
+  cudaStream_t st;
+  int saved_nseg;
+  int64_t saved_rows[MAX_SEGMENTS + 1];
+  explicit HostPipeGuard(acspgemm_plan p, cudaStream_t s) : plan(p), st(s), saved_nseg(p->nseg_explicit) {
+    for (int i = 0; i <= MAX_SEGMENTS; ++i) saved_rows[i] = p->seg_rows_explicit[i];
+  }
+  ~HostPipeGuard() {
+    if (plan->hp_cs) cudaStreamSynchronize(plan->hp_cs);
+    cudaStreamSynchronize(st);
+    plan->nseg_explicit = saved_nseg;
+    for (int i = 0; i <= MAX_SEGMENTS; ++i) plan->seg_rows_explicit[i] = saved_rows[i];
+  }
+};
+
 template <typename P>
 struct Scratch {
   P* d = nullptr;
@@ -575,7 +609,8 @@ acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options
     return set_err(ACSPGEMM_ERR_INVALID_ARG, "num_segments > 64");
   }
   std::memset(&p->info, 0, sizeof(p->info));
-  cudaError_t e = cudaHostAlloc(&p->h_scal, sizeof(int64_t) * 32, cudaHostAllocDefault);
+  // mapped: read-backs are written by a kernel (launch_read_back), not a copy engine
+  cudaError_t e = cudaHostAlloc(&p->h_scal, sizeof(int64_t) * H_SCAL_WORDS, cudaHostAllocMapped);
   if (e != cudaSuccess) {
     delete p;
     return set_err(ACSPGEMM_ERR_CUDA, std::string("cudaHostAlloc: ") + cudaGetErrorString(e));
@@ -597,6 +632,15 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
                   &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
                   &p->cur_last, &p->err, &p->bused, &p->bused_scan};
   for (DevBuf* b : bs) free_buf(*b);
+  for (int i = 0; i < 3; ++i) {
+    free_buf(p->hp_a[i]);
+    free_buf(p->hp_b[i]);
+    free_buf(p->hp_c[0][i]);
+    free_buf(p->hp_c[1][i]);
+  }
+  if (p->hp_cs) cudaStreamDestroy(p->hp_cs);
+  if (p->hp_ready) cudaEventDestroy(p->hp_ready);
+  for (cudaEvent_t e : p->hp_copied) if (e) cudaEventDestroy(e);
   if (p->h_scal) cudaFreeHost(p->h_scal);
   if (p->ev_ok)
     for (int i = 0; i < NSTAGE_EV; ++i) cudaEventDestroy(p->ev[i]);
@@ -685,6 +729,118 @@ acspgemm_status acspgemm_rap(const acspgemm_csr_in* R, const acspgemm_csr_in* A,
   acspgemm_free_csr(&AP, stream);
   if (s == ACSPGEMM_OK) ACS_CUDA(cudaStreamSynchronize(reinterpret_cast<cudaStream_t>(stream)));
   return s;
+}
+
+acspgemm_status acspgemm_multiply_host(acspgemm_plan p, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
+                                       acspgemm_dtype dtype, void* stream, int npieces, acspgemm_csr_out* C,
+                                       int64_t capacity) {
+  if (!p) return set_err(ACSPGEMM_ERR_INVALID_ARG, "plan is NULL");
+  acspgemm_status s;
+  if ((s = check_in(A, "A")) != ACSPGEMM_OK) return s;
+  if ((s = check_in(B, "B")) != ACSPGEMM_OK) return s;
+  if (!C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C is NULL");
+  if (dtype != ACSPGEMM_F32 && dtype != ACSPGEMM_F64) return set_err(ACSPGEMM_ERR_INVALID_ARG, "bad dtype");
+  if (A->cols != B->rows) return set_err(ACSPGEMM_ERR_DIM_MISMATCH, "A.cols != B.rows");
+  const int S = p->opt.num_segments;
+  if (npieces < 1 || npieces > S) return set_err(ACSPGEMM_ERR_INVALID_ARG, "npieces must be in [1, num_segments]");
+  if (capacity < 0 || (capacity > 0 && (!C->col_idx || !C->val)))
+    return set_err(ACSPGEMM_ERR_INVALID_ARG, "bad C capacity / buffers");
+  if (!C->row_ptr) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C.row_ptr is NULL");
+  const size_t vb = dtype == ACSPGEMM_F64 ? 8 : 4;
+  C->rows = A->rows;
+  C->cols = B->cols;
+  C->nnz = 0;
+  if (A->rows == 0) { C->row_ptr[0] = 0; return ACSPGEMM_OK; }
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  HostPipeGuard guard(p, st);
+  if (!p->hp_cs) ACS_CUDA(cudaStreamCreateWithFlags(&p->hp_cs, cudaStreamNonBlocking));
+  if (!p->hp_ready) ACS_CUDA(cudaEventCreateWithFlags(&p->hp_ready, cudaEventDisableTiming));
+  for (cudaEvent_t& e : p->hp_copied)
+    if (!e) ACS_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  // inputs host -> device into plan memory (B once when it is A)
+  const bool same = B->row_ptr == A->row_ptr && B->col_idx == A->col_idx && B->val == A->val &&
+                    B->rows == A->rows && B->nnz == A->nnz;
+  const acspgemm_csr_in* M[2] = {A, B};
+  DevBuf* Dm[2] = {p->hp_a, p->hp_b};
+  acspgemm_csr_in D[2];
+  for (int m = 0; m < (same ? 1 : 2); ++m) {
+    const acspgemm_csr_in* H = M[m];
+    DevBuf* d = Dm[m];
+    const int64_t base = H->rows > 0 ? H->row_ptr[0] : 0;
+    ACS_ENSURE(d[0], sizeof(int32_t) * (H->rows + 1));
+    ACS_ENSURE(d[1], sizeof(int32_t) * H->nnz);
+    ACS_ENSURE(d[2], vb * H->nnz);
+    ACS_CUDA(cudaMemcpyAsync(d[0].p, H->row_ptr, sizeof(int32_t) * (H->rows + 1), cudaMemcpyHostToDevice, st));
+    if (H->nnz > 0) {
+      ACS_CUDA(cudaMemcpyAsync(d[1].p, H->col_idx + base, sizeof(int32_t) * H->nnz, cudaMemcpyHostToDevice, st));
+      ACS_CUDA(cudaMemcpyAsync(d[2].p, static_cast<const char*>(H->val) + vb * base, vb * H->nnz,
+                               cudaMemcpyHostToDevice, st));
+    }
+    // device view: row_ptr values index col / val directly (base shifted away)
+    D[m] = acspgemm_csr_in{H->rows, H->cols, H->nnz, ptr<const int32_t>(d[0]), ptr<const int32_t>(d[1]) - base,
+                           static_cast<const char*>(d[2].p) - vb * base};
+  }
+  if (same) D[1] = D[0];
+  // canonical segments of the whole A (plan memory, one read-back), grouped into pieces
+  int64_t seg[MAX_SEGMENTS + 1];
+  {
+    ACS_ENSURE(p->seg, sizeof(int64_t) * (4 * (MAX_SEGMENTS + 1) + 2));
+    int64_t* sd = ptr<int64_t>(p->seg);
+    const CsrView Av{D[0].rows, D[0].cols, D[0].row_ptr, D[0].col_idx, D[0].val};
+    launch_segments(Av, S, nullptr, sd, reinterpret_cast<int32_t*>(sd + 4 * (MAX_SEGMENTS + 1)), st);
+    tl_launches += 1;
+    ACS_CUDA(cudaGetLastError());
+    ACS_CUDA(cudaMemcpyAsync(seg, sd, sizeof(int64_t) * (S + 1), cudaMemcpyDeviceToHost, st));
+    ACS_CUDA(cudaStreamSynchronize(st));
+  }
+  int64_t off = 0;
+  bool overflow = false;
+  for (int g = 0; g < npieces; ++g) {
+    const int s0 = (int)((int64_t)g * S / npieces), s1 = (int)((int64_t)(g + 1) * S / npieces);
+    const int64_t r0 = seg[s0], r1 = seg[s1];
+    p->nseg_explicit = s1 - s0;
+    for (int i = 0; i <= s1 - s0; ++i) p->seg_rows_explicit[i] = seg[s0 + i] - r0;
+    const acspgemm_csr_in V{r1 - r0, A->cols, (int64_t)A->row_ptr[r1] - A->row_ptr[r0], D[0].row_ptr + r0,
+                            D[0].col_idx, D[0].val};
+    int64_t nnz_g = 0;
+    if ((s = symbolic_impl(p, &V, &D[1], dtype, st, &nnz_g)) != ACSPGEMM_OK) return s;
+    if (off + nnz_g >= (int64_t(1) << 31)) return set_err(ACSPGEMM_ERR_INDEX_OVERFLOW, "nnz(C) >= 2^31");
+    if (off + nnz_g > capacity) overflow = true;
+    if (!overflow) {
+      // piece buffer k alternates; its previous copy-out (piece g - 2) must be done
+      DevBuf* cb = p->hp_c[g & 1];
+      ACS_CUDA(cudaStreamWaitEvent(st, p->hp_copied[g & 1], 0));
+      if (cb[0].bytes < sizeof(int32_t) * (V.rows + 1) || cb[1].bytes < sizeof(int32_t) * nnz_g ||
+          cb[2].bytes < vb * nnz_g)
+        ACS_CUDA(cudaEventSynchronize(p->hp_copied[g & 1]));   // about to re-allocate it
+      ACS_ENSURE(cb[0], sizeof(int32_t) * (V.rows + 1));
+      ACS_ENSURE(cb[1], sizeof(int32_t) * nnz_g);
+      ACS_ENSURE(cb[2], vb * nnz_g);
+      acspgemm_csr_out Cg{V.rows, B->cols, nnz_g, ptr<int32_t>(cb[0]), ptr<int32_t>(cb[1]), cb[2].p};
+      if ((s = numeric_impl(p, &Cg, st, (int32_t)off)) != ACSPGEMM_OK) return s;
+      ACS_CUDA(cudaGetLastError());
+      // copy piece g out on the copy stream while piece g + 1 is multiplied
+      ACS_CUDA(cudaEventRecord(p->hp_ready, st));
+      ACS_CUDA(cudaStreamWaitEvent(p->hp_cs, p->hp_ready, 0));
+      // (the size queries of later pieces read back through mapped memory, never through
+      // a copy engine, so they do not queue behind these copies)
+      ACS_CUDA(cudaMemcpyAsync(C->row_ptr + r0, Cg.row_ptr, sizeof(int32_t) * (V.rows + 1), cudaMemcpyDeviceToHost,
+                               p->hp_cs));
+      if (nnz_g > 0) {
+        ACS_CUDA(cudaMemcpyAsync(C->col_idx + off, Cg.col_idx, sizeof(int32_t) * nnz_g, cudaMemcpyDeviceToHost,
+                                 p->hp_cs));
+        ACS_CUDA(cudaMemcpyAsync(static_cast<char*>(C->val) + vb * off, Cg.val, vb * nnz_g, cudaMemcpyDeviceToHost,
+                                 p->hp_cs));
+      }
+      ACS_CUDA(cudaEventRecord(p->hp_copied[g & 1], p->hp_cs));
+    }
+    off += nnz_g;
+  }
+  ACS_CUDA(cudaStreamSynchronize(p->hp_cs));
+  C->nnz = off;
+  if (overflow) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C capacity " + std::to_string(capacity) +
+                                                         " < nnz(C) = " + std::to_string(off));
+  return ACSPGEMM_OK;
 }
 
 acspgemm_status acspgemm_free_csr(acspgemm_csr_out* C, void* stream) {

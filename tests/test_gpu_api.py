@@ -191,3 +191,37 @@ def test_rap_galerkin(cuda_available):
     assert (rp == A4.row_ptr).all() and (col == A4.col).all() and (val == 4 * A4.val).all()
     rp, col, val = p.rap_lib_alloc(dev(R), dev(A), dev(P))
     assert (rp == A4.row_ptr).all() and (col == A4.col).all() and (val == 4 * A4.val).all()
+
+
+@pytest.mark.parametrize("pieces", [1, 3, 8])
+def test_multiply_host_pieces_bit_identical(pieces, cuda_available):
+    """acspgemm_multiply_host: host in, host out, pipelined over canonical-segment pieces;
+    C equals the device multiply byte for byte and the oracle within tolerance."""
+    p = pkg()
+    A = power_law_csr(4000, 4000, 10, 1.3, 1200, seed=31)
+    full = p.multiply(dev(A), dev(A))
+    frp, fcol, fval = full.to_numpy()
+    rp, col, val = p.multiply_host(A, A, pieces=pieces)
+    assert (rp.numpy() == frp).all() and (col.numpy() == fcol).all()
+    assert val.numpy().tobytes() == fval.tobytes()
+    ref = oracle.gustavson(A, A)
+    assert (np.abs(val.numpy() - ref.val) <= 1e-12 * ref.absval).all()
+
+
+def test_multiply_host_rectangular_capacity(cuda_available):
+    """B distinct from A (copied separately), numpy buffers, capacity overflow reports nnz."""
+    p = pkg()
+    A = random_csr(300, 500, 0.02, seed=41)
+    B = random_csr(500, 200, 0.03, seed=42)
+    ref = oracle.gustavson(A, B)
+    nnz = int(ref.row_ptr[-1])
+    plan = p.Plan()
+    small = (np.zeros(301, np.int32), np.zeros(max(nnz - 1, 1), np.int32), np.zeros(max(nnz - 1, 1)))
+    with pytest.raises(p.AcspgemmError):
+        plan.multiply_host(A, B, out=small, pieces=2)
+    out = (np.zeros(301, np.int32), np.zeros(nnz + 5, np.int32), np.zeros(nnz + 5))
+    rp, col, val = plan.multiply_host(A, B, out=out, pieces=2)
+    assert (rp == ref.row_ptr).all() and (col == ref.col).all()
+    assert (np.abs(val - ref.val) <= 1e-12 * ref.absval).all()
+    # the plan's own segmentation is restored afterwards
+    check(plan.multiply(dev(A), dev(B)), A, B)
