@@ -35,6 +35,8 @@ constexpr int RADIX_BITS = ACS_RADIX_BITS;   // digit width of one radix-sort pa
 constexpr int DEFAULT_SEGMENTS = 8;          // canonical segments
 constexpr int MAX_SEGMENTS = 64;
 constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)
+constexpr int SEARCH_MAXP = 1024;            // Search Merge limit; longer chunk lists: dense slices (R30)
+constexpr int GIANT_SLICE = 4096;            // columns per dense-slice CTA
 constexpr int PAIR_MAX = 512;                // two-chunk rows up to this size: warp merge
 static_assert((1 << IDXBITS) == CAP, "IDXBITS must be log2(CAP)");
 static_assert(KEEP <= CAP / 2, "kept row must leave room for new products");
@@ -60,7 +62,7 @@ struct SharedRow {
   int32_t total;          // sum of the row's element counts over its chunks (pre-merge)
   int64_t merge_off;      // where the merged row goes in the merge pool
   int32_t merged;         // merged element count (written by the merge kernels)
-  int32_t kind;           // 0 multi (block), 1 path, 2 search, 3 multi (warp pair)
+  int32_t kind;           // 0 multi (block), 1 path, 2 search, 3 multi (warp pair), 4 dense slices
 };
 
 // ---------------------------------------------------------------- helpers --

@@ -64,6 +64,7 @@ struct MergeState {
   int32_t* shared_flag;          // [max_chunks] 1 where a shared row starts
   int64_t* shared_pos;           // [max_chunks] exclusive scan of shared_flag
   SharedRow* shared;             // [max_chunks]
+  const int32_t* pool_col;       // chunk columns (row spans for the merge classification)
   int64_t* scan_tmp;
 };
 void launch_gather_chunks(const MergeState& m, cudaStream_t st);
@@ -78,7 +79,8 @@ struct MergeLists {
   int32_t* path_idx;
   int32_t* search_idx;
   int32_t* pair_idx;             // two-chunk rows of <= PAIR_MAX elements (warp merge)
-  int64_t* counts_dev;           // [8]: nmulti, npath, nsearch, npair, merge_total, -, multi_total
+  int32_t* giant_idx;            // rows of > SEARCH_MAXP chunks (dense slices)
+  int64_t* counts_dev;           // [8]: nmulti, npath, nsearch, npair, merge_total, ngiant, multi_total
   int64_t* merge_total_scan;     // [nshared] exclusive scan of totals -> merge offsets
   int64_t* multi_scan;           // [nshared]
   int32_t* group_of;             // [nshared]
@@ -109,6 +111,18 @@ void launch_multi_merge(const MergeArgs& a, bool f64, cudaStream_t st);
 void launch_pair_merge(const MergeArgs& a, bool f64, cudaStream_t st);
 void launch_path_merge(const MergeArgs& a, bool f64, cudaStream_t st);
 void launch_search_merge(const MergeArgs& a, bool f64, cudaStream_t st);
+struct GiantArgs {                // dense-slice merge of rows with > SEARCH_MAXP chunks
+  const int32_t* list;            // [n] indices into shared
+  int64_t n;
+  int32_t* glo;                   // [n] first column of the row's span
+  int64_t* gnsl;                  // [n] slices of the row
+  int64_t* gbase;                 // [n] exclusive scan of gnsl
+  int32_t* tcol;                  // [nslices * GIANT_SLICE] per-slice outputs
+  void* tval;
+  int32_t* tcnt;                  // [nslices]
+};
+void launch_giant_span(const MergeArgs& a, const GiantArgs& g, cudaStream_t st);
+void launch_giant_merge(const MergeArgs& a, const GiantArgs& g, int64_t nslices, bool f64, cudaStream_t st);
 
 // ---- stage 4: chunk copy (copy.cu) ----------------------------------------------
 struct CopyArgs {

@@ -73,6 +73,7 @@ struct acspgemm_plan_s {
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan;
+  DevBuf lgiant, g_lo, g_nsl, g_base, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30)
   // acspgemm_multiply_host: device copies of A and B, two C piece buffers, copy stream
   DevBuf hp_a[3], hp_b[3], hp_c[2][3];
   cudaStream_t hp_cs = nullptr;
@@ -322,6 +323,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ms.shared_flag = ptr<int32_t>(p->sflag);
   ms.shared_pos = ptr<int64_t>(p->spos);
   ms.shared = ptr<SharedRow>(p->shared);
+  ms.pool_col = ptr<int32_t>(p->pool_col);
   ms.scan_tmp = ptr<int64_t>(p->scan_tmp);
   launch_gather_chunks(ms, st);
   launch_find_shared(ms, scal + 4, st);
@@ -335,7 +337,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   p->info.nshared = p->nshared;
   p->info.chunk_elems = p->h_scal[2];
   const int64_t nsh = p->nshared;
-  int64_t nmulti = 0, npath = 0, nsearch = 0, npair = 0, merge_total = 0, ngroups = 0;
+  int64_t nmulti = 0, npath = 0, nsearch = 0, npair = 0, merge_total = 0, ngroups = 0, ngiant = 0;
   if (nsh > 0) {
     ACS_ENSURE(p->kflag, sizeof(int32_t) * nsh);
     ACS_ENSURE(p->kpos, sizeof(int64_t) * nsh);
@@ -343,6 +345,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     ACS_ENSURE(p->lpath, sizeof(int32_t) * nsh);
     ACS_ENSURE(p->lsearch, sizeof(int32_t) * nsh);
     ACS_ENSURE(p->lpair, sizeof(int32_t) * nsh);
+    ACS_ENSURE(p->lgiant, sizeof(int32_t) * nsh);
     ACS_ENSURE(p->mtscan, sizeof(int64_t) * nsh);
     ACS_ENSURE(p->mscan, sizeof(int64_t) * nsh);
     ACS_ENSURE(p->group_of, sizeof(int32_t) * nsh);
@@ -355,6 +358,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     L.path_idx = ptr<int32_t>(p->lpath);
     L.search_idx = ptr<int32_t>(p->lsearch);
     L.pair_idx = ptr<int32_t>(p->lpair);
+    L.giant_idx = ptr<int32_t>(p->lgiant);
     L.counts_dev = scal + 8;
     L.merge_total_scan = ptr<int64_t>(p->mtscan);
     L.multi_scan = ptr<int64_t>(p->mscan);
@@ -362,14 +366,15 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     L.group_start = nullptr;
     L.scan_tmp = ptr<int64_t>(p->scan_tmp);
     launch_classify(L, st);
-    tl_launches += 4 * 5 + 1 + 3 + 1;
+    tl_launches += 5 * 5 + 1 + 3 + 1;
     ACS_CUDA(cudaGetLastError());
-    if ((s = sync_read(p, scal + 8, 5, st)) != ACSPGEMM_OK) return s;
+    if ((s = sync_read(p, scal + 8, 6, st)) != ACSPGEMM_OK) return s;
     nmulti = p->h_scal[0];
     npath = p->h_scal[1];
     nsearch = p->h_scal[2];
     npair = p->h_scal[3];
     merge_total = p->h_scal[4];
+    ngiant = p->h_scal[5];
     // Multi-Merge packing needs the multi totals: scan them over the multi list
     if (nmulti > 0) {
       // upper bound of groups from merge_total (multi totals <= merge_total)
@@ -413,6 +418,32 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     ma.list = ptr<int32_t>(p->lsearch);
     ma.nlist = nsearch;
     if (nsearch > 0) { launch_search_merge(ma, p->f64, st); tl_launches += 1; }
+    if (ngiant > 0) {
+      // rows of > SEARCH_MAXP chunks: dense column slices (reading R30)
+      ACS_ENSURE(p->g_lo, sizeof(int32_t) * ngiant);
+      ACS_ENSURE(p->g_nsl, sizeof(int64_t) * ngiant);
+      ACS_ENSURE(p->g_base, sizeof(int64_t) * ngiant);
+      GiantArgs g;
+      g.list = ptr<int32_t>(p->lgiant);
+      g.n = ngiant;
+      g.glo = ptr<int32_t>(p->g_lo);
+      g.gnsl = ptr<int64_t>(p->g_nsl);
+      g.gbase = ptr<int64_t>(p->g_base);
+      launch_giant_span(ma, g, st);
+      launch_scan_i64(g.gnsl, g.gbase, ngiant, scal + 24, ptr<int64_t>(p->scan_tmp), st);
+      tl_launches += 1 + 3;
+      ACS_CUDA(cudaGetLastError());
+      if ((s = sync_read(p, scal + 24, 1, st)) != ACSPGEMM_OK) return s;
+      const int64_t nslices = p->h_scal[0];
+      ACS_ENSURE(p->g_tcol, sizeof(int32_t) * nslices * GIANT_SLICE);
+      ACS_ENSURE(p->g_tval, (size_t)vbytes * nslices * GIANT_SLICE);
+      ACS_ENSURE(p->g_tcnt, sizeof(int32_t) * nslices);
+      g.tcol = ptr<int32_t>(p->g_tcol);
+      g.tval = p->g_tval.p;
+      g.tcnt = ptr<int32_t>(p->g_tcnt);
+      launch_giant_merge(ma, g, nslices, p->f64, st);
+      tl_launches += 2;
+    }
     ACS_CUDA(cudaGetLastError());
   } else {
     record(p, S_MM, st);
@@ -421,7 +452,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   }
   p->info.nmulti = nmulti + npair;
   p->info.npath = npath;
-  p->info.nsearch = nsearch;
+  p->info.nsearch = nsearch + ngiant;
   p->info.nmulti_groups = ngroups;
   p->info.merge_elems = merge_total;
 
@@ -630,7 +661,8 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
                   &p->descs, &p->dense, &p->sflag, &p->spos, &p->shared, &p->row_count, &p->row_ptr,
                   &p->scan_tmp, &p->kflag, &p->kpos, &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan,
                   &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
-                  &p->cur_last, &p->err, &p->bused, &p->bused_scan};
+                  &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->lgiant, &p->g_lo, &p->g_nsl,
+                  &p->g_base, &p->g_tcol, &p->g_tval, &p->g_tcnt};
   for (DevBuf* b : bs) free_buf(*b);
   for (int i = 0; i < 3; ++i) {
     free_buf(p->hp_a[i]);

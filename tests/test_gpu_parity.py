@@ -133,7 +133,9 @@ def test_path_merge_windows_dense_columns(ncols_log2, cuda_available):
     r = np.repeat(np.arange(rows), k)
     c = np.concatenate([np.sort(rng.choice(6000, k, replace=False)) for _ in range(rows)])
     A = from_coo(rows, 6000, r, c, rng.uniform(-1, 1, rows * k))
-    B = random_rowlen_csr(6000, n, np.full(6000, 20), seed=ncols_log2, values="uniform")
+    # 1500 x 5 = 7,500 products per row: several chunks, at most 4 windows (Path Merge;
+    # longer dense rows go to the dense slices of reading R30)
+    B = random_rowlen_csr(6000, n, np.full(6000, 5), seed=ncols_log2, values="uniform")
     plan = pkg().Plan()
     assert_parity(A, B, np.float64, plan=plan)
     assert plan.info()["npath"] >= 1
@@ -157,6 +159,23 @@ def test_path_merge_window_all_ones_key(cuda_available):
     assert_parity(A, B, np.float64, plan=plan)
     info = plan.info()
     assert info["npath"] == 1 and info["nchunks"] == 3
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_giant_row_dense_slices(dt, cuda_available):
+    """A row gathering 2.2M products over a 200K-column range is split into more than
+    SEARCH_MAXP chunks and merged by dense column slices (reading R30); small rows and an
+    empty row around it take the other paths."""
+    n_b, ncol = 70000, 200000
+    rng = np.random.default_rng(17)
+    rows = [0] * n_b + [1, 1, 3]
+    cols = list(range(n_b)) + [5, 9, 11]
+    A = from_coo(4, n_b, rows, cols, rng.uniform(-1, 1, len(rows)))
+    B = random_rowlen_csr(n_b, ncol, np.full(n_b, 32), seed=18, values="uniform")
+    plan = pkg().Plan()
+    assert_parity(A, B, dt, plan=plan)
+    info = plan.info()
+    assert info["nsearch"] >= 1 and info["nchunks"] > 1024
 
 
 def test_dense_row_search_merge(cuda_available):
