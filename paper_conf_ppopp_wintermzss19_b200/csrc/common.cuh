@@ -37,6 +37,7 @@ constexpr int MAX_SEGMENTS = 64;
 constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)
 constexpr int SEARCH_MAXP = 1024;            // Search Merge limit; longer chunk lists: dense slices (R30)
 constexpr int GIANT_SLICE = 4096;            // columns per dense-slice CTA
+constexpr int DENSE_SPAN_RATIO = 16;         // dense slices when span <= 16 x pre-merge elements
 constexpr int PAIR_MAX = 512;                // two-chunk rows up to this size: warp merge
 static_assert((1 << IDXBITS) == CAP, "IDXBITS must be log2(CAP)");
 static_assert(KEEP <= CAP / 2, "kept row must leave room for new products");

@@ -117,11 +117,12 @@ struct GiantArgs {                // dense-slice merge of rows with > SEARCH_MAX
   int32_t* glo;                   // [n] first column of the row's span
   int64_t* gnsl;                  // [n] slices of the row
   int64_t* gbase;                 // [n] exclusive scan of gnsl
-  int32_t* tcol;                  // [nslices * GIANT_SLICE] per-slice outputs
-  void* tval;
-  int32_t* tcnt;                  // [nslices]
+  int32_t* gent;                  // [nslices] pre-merge entries per slice
+  int64_t* gpos;                  // [nslices] exclusive scan of gent
+  int32_t* tcnt;                  // [nslices] merged entries per slice
 };
 void launch_giant_span(const MergeArgs& a, const GiantArgs& g, cudaStream_t st);
+void launch_giant_count(const MergeArgs& a, const GiantArgs& g, int64_t nslices, cudaStream_t st);
 void launch_giant_merge(const MergeArgs& a, const GiantArgs& g, int64_t nslices, bool f64, cudaStream_t st);
 
 // ---- stage 4: chunk copy (copy.cu) ----------------------------------------------

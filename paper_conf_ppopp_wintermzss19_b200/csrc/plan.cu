@@ -73,7 +73,7 @@ struct acspgemm_plan_s {
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan;
-  DevBuf lgiant, g_lo, g_nsl, g_base, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30)
+  DevBuf lgiant, g_lo, g_nsl, g_base, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30): lists, spans, slices
   // acspgemm_multiply_host: device copies of A and B, two C piece buffers, copy stream
   DevBuf hp_a[3], hp_b[3], hp_c[2][3];
   cudaStream_t hp_cs = nullptr;
@@ -435,14 +435,17 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
       ACS_CUDA(cudaGetLastError());
       if ((s = sync_read(p, scal + 24, 1, st)) != ACSPGEMM_OK) return s;
       const int64_t nslices = p->h_scal[0];
-      ACS_ENSURE(p->g_tcol, sizeof(int32_t) * nslices * GIANT_SLICE);
-      ACS_ENSURE(p->g_tval, (size_t)vbytes * nslices * GIANT_SLICE);
+      ACS_ENSURE(p->g_tcol, sizeof(int32_t) * nslices);            // entries per slice
+      ACS_ENSURE(p->g_tval, sizeof(int64_t) * nslices);            // their scan
       ACS_ENSURE(p->g_tcnt, sizeof(int32_t) * nslices);
-      g.tcol = ptr<int32_t>(p->g_tcol);
-      g.tval = p->g_tval.p;
+      ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * scan_tmp_elems(nslices + 1));
+      g.gent = ptr<int32_t>(p->g_tcol);
+      g.gpos = ptr<int64_t>(p->g_tval);
       g.tcnt = ptr<int32_t>(p->g_tcnt);
+      launch_giant_count(ma, g, nslices, st);
+      launch_scan_i32(g.gent, g.gpos, nslices, scal + 25, ptr<int64_t>(p->scan_tmp), st);
       launch_giant_merge(ma, g, nslices, p->f64, st);
-      tl_launches += 2;
+      tl_launches += 1 + 3 + 2;
     }
     ACS_CUDA(cudaGetLastError());
   } else {
