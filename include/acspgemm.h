@@ -83,7 +83,13 @@ typedef struct {
   int validate_inputs;       /* 1: check that A and B are canonical CSR (one extra sync) */
   int collect_stage_times;   /* 1: record CUDA events between stages (acspgemm_stage_times) */
   int num_segments;          /* canonical segments S (default 8, max 64) */
+  int strategy;              /* ACSPGEMM_STRATEGY_ADAPTIVE (default): each block is tried by the
+                                hash accumulator first and falls back to AC-ESC (reading R31);
+                                ACSPGEMM_STRATEGY_ESC: every block through AC-ESC */
 } acspgemm_options;
+
+#define ACSPGEMM_STRATEGY_ADAPTIVE 0
+#define ACSPGEMM_STRATEGY_ESC 1
 
 /* Counters of the last multiply of a plan (host values). */
 typedef struct {
@@ -101,9 +107,10 @@ typedef struct {
   int64_t kernel_launches;   /* kernels launched by the last symbolic + numeric */
   int32_t nsegments;
   int64_t segment_rows[65];
+  int64_t nhash_blocks;      /* blocks completed by the hash accumulator (strategy ADAPTIVE) */
 } acspgemm_info;
 
-/* Defaults: no pool limit, no validation, no stage times, 8 segments. */
+/* Defaults: no pool limit, no validation, no stage times, 8 segments, adaptive strategy. */
 void acspgemm_options_default(acspgemm_options* opt);
 
 /* Create a plan.  opt may be NULL (defaults).  *plan receives the handle. */
@@ -170,8 +177,9 @@ acspgemm_status acspgemm_rap(const acspgemm_csr_in* R, const acspgemm_csr_in* A,
 acspgemm_status acspgemm_free_csr(acspgemm_csr_out* C, void* stream);
 
 /* Per-stage device times (ms) of the last symbolic + numeric when collect_stage_times
- * was set, in the order of Fig. 7 (L740): GLB, ESC, MCC, MM, PM, SM, SCAN, CC.
- * Writes min(n, 8) values.  Synchronises the plan's events. */
+ * was set, in the order of Fig. 7 (L740): GLB, ESC, MCC, MM, PM, SM, SCAN, CC, then HASH:
+ * the part of ESC spent in the hash accumulator (strategy ADAPTIVE, reading R31).
+ * Writes min(n, 9) values.  Synchronises the plan's events. */
 acspgemm_status acspgemm_stage_times(acspgemm_plan plan, float* ms_out, int n);
 
 /* Counters of the last multiply. */

@@ -29,7 +29,8 @@ class CsrOut(ctypes.Structure):
 
 class Options(ctypes.Structure):
     _fields_ = [("pool_limit_bytes", ctypes.c_size_t), ("validate_inputs", ctypes.c_int),
-                ("collect_stage_times", ctypes.c_int), ("num_segments", ctypes.c_int)]
+                ("collect_stage_times", ctypes.c_int), ("num_segments", ctypes.c_int),
+                ("strategy", ctypes.c_int)]
 
 
 class Info(ctypes.Structure):
@@ -37,7 +38,8 @@ class Info(ctypes.Structure):
                 ("chunk_elems", I64), ("nshared", I64), ("nmulti", I64), ("npath", I64),
                 ("nsearch", I64), ("nmulti_groups", I64), ("merge_elems", I64),
                 ("pool_bytes", I64), ("helper_bytes", I64), ("pool_estimate_bytes", ctypes.c_double),
-                ("kernel_launches", I64), ("nsegments", I32), ("segment_rows", I64 * 65)]
+                ("kernel_launches", I64), ("nsegments", I32), ("segment_rows", I64 * 65),
+                ("nhash_blocks", I64)]
 
 
 # name -> (restype, argtypes); every symbol include/acspgemm.h declares

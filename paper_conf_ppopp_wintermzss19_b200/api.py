@@ -16,7 +16,7 @@ from . import _lib
 from ._lib import CsrIn, CsrOut, Info, Options, check, load
 
 F32, F64 = 0, 1
-STAGES = ("GLB", "ESC", "MCC", "MM", "PM", "SM", "SCAN", "CC")
+STAGES = ("GLB", "ESC", "MCC", "MM", "PM", "SM", "SCAN", "CC", "HASH")   # HASH: k_hash part of ESC
 
 
 @dataclass
@@ -85,7 +85,11 @@ class Plan:
     """A reusable multiply plan (owns the chunk pool and helper memory)."""
 
     def __init__(self, pool_limit_bytes: int = 0, validate: bool = False, stage_times: bool = False,
-                 num_segments: int = 8):
+                 num_segments: int = 8, strategy: str = "adaptive"):
+        """strategy: "adaptive" (hash accumulator per block, AC-ESC fallback; reading R31)
+        or "esc" (every block through AC-ESC)."""
+        if strategy not in ("adaptive", "esc"):
+            raise ValueError("strategy must be 'adaptive' or 'esc'")
         lib = load()
         opt = Options()
         lib.acspgemm_options_default(ctypes.byref(opt))
@@ -93,6 +97,7 @@ class Plan:
         opt.validate_inputs = int(bool(validate))
         opt.collect_stage_times = int(bool(stage_times))
         opt.num_segments = int(num_segments)
+        opt.strategy = 0 if strategy == "adaptive" else 1
         h = ctypes.c_void_p()
         check(lib.acspgemm_plan_create(ctypes.byref(h), ctypes.byref(opt)), "acspgemm_plan_create")
         self._h = h
@@ -192,8 +197,8 @@ class Plan:
         return d
 
     def stage_times(self) -> dict:
-        buf = (ctypes.c_float * 8)()
-        check(self._lib.acspgemm_stage_times(self._h, buf, 8), "acspgemm_stage_times")
+        buf = (ctypes.c_float * len(STAGES))()
+        check(self._lib.acspgemm_stage_times(self._h, buf, len(STAGES)), "acspgemm_stage_times")
         return {k: float(buf[i]) for i, k in enumerate(STAGES)}
 
     def block_row_starts(self) -> np.ndarray:

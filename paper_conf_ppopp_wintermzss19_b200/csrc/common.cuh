@@ -38,7 +38,19 @@ constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)
 constexpr int SEARCH_MAXP = 1024;            // Search Merge limit; longer chunk lists: dense slices (R30)
 constexpr int GIANT_SLICE = 4096;            // columns per dense-slice CTA
 constexpr int DENSE_SPAN_RATIO = 16;         // dense slices when span <= 16 x pre-merge elements
-constexpr int PAIR_MAX = 512;                // two-chunk rows up to this size: warp merge
+constexpr int PAIR_MAX = 512;
+// hash accumulator (hash.cu, reading R31)
+constexpr int HASH_WARPS = 4;                // warps per CTA; each emits one chunk per block
+constexpr int HASH_THREADS = 32 * HASH_WARPS;
+constexpr int HASH_T = 512;                  // table slots per warp
+constexpr int HASH_UMAX = 256;               // max distinct columns of a row (load <= 1/2)
+#ifndef ACS_HASH_PROWMAX
+#define ACS_HASH_PROWMAX 2048
+#endif
+constexpr int HASH_PROWMAX = ACS_HASH_PROWMAX; // blocks with a longer row (in products) go to AC-ESC
+#ifndef HASH_MIN_BLOCKS
+#define HASH_MIN_BLOCKS 5
+#endif                // two-chunk rows up to this size: warp merge
 static_assert((1 << IDXBITS) == CAP, "IDXBITS must be log2(CAP)");
 static_assert(KEEP <= CAP / 2, "kept row must leave room for new products");
 static_assert(NPB % THREADS == 0, "NPB must be a multiple of THREADS");

@@ -224,6 +224,7 @@ __global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
   EscSmem<T>& S = *reinterpret_cast<EscSmem<T>*>(smem_raw);
   const int tid = threadIdx.x;
   const int b = blockIdx.x;
+  if (a.hash_done && a.hash_done[b]) return;        // finished by the hash accumulator (R31)
   const int32_t* __restrict__ arp = a.A.row_ptr;
   const int32_t* __restrict__ acol = a.A.col;
   const T* __restrict__ aval = reinterpret_cast<const T*>(a.A.val);

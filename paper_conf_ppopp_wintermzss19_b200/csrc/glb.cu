@@ -101,7 +101,8 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
                                const int32_t* __restrict__ brp, int nseg, const int64_t* __restrict__ seg,
                                const int32_t* __restrict__ nblocks_dev, int64_t max_blocks,
                                int32_t* __restrict__ nz_begin, int32_t* __restrict__ nz_end,
-                               int64_t* __restrict__ products, int64_t* __restrict__ slots) {
+                               int64_t* __restrict__ products, int64_t* __restrict__ slots,
+                               int32_t* __restrict__ hash_ok) {
   __shared__ int64_t s_nz[SEG_STRIDE], s_base[SEG_STRIDE];
   for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
     s_nz[i] = seg[SEG_STRIDE + i];
@@ -113,23 +114,36 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
   if (b >= max_blocks) return;
   const int nblocks = *nblocks_dev;
   if (b >= nblocks) {
-    if (lane == 0) { products[b] = 0; slots[b] = 0; nz_begin[b] = 0; nz_end[b] = 0; }
+    if (lane == 0) {
+      products[b] = 0; slots[b] = 0; nz_begin[b] = 0; nz_end[b] = 0;
+      if (hash_ok) hash_ok[b] = 0;
+    }
     return;
   }
   int s = 0;
   while (s + 1 < nseg && s_base[s + 1] <= b) ++s;
   const int64_t nzb = s_nz[s] + (b - s_base[s]) * NPB;
   const int64_t nze = min(nzb + (int64_t)NPB, s_nz[s + 1]);
-  int64_t sum = 0;
+  int64_t sum = 0, waves = 0;
   for (int64_t p = nzb + lane; p < nze; p += 32) {
     const int k = acol[p];
-    sum += brp[k + 1] - brp[k];
+    const int len = brp[k + 1] - brp[k];
+    sum += len;
+    waves += (len + 31) >> 5;
   }
 #pragma unroll
-  for (int d = 16; d > 0; d >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, d);
+  for (int d = 16; d > 0; d >>= 1) {
+    sum += __shfl_xor_sync(0xffffffffu, sum, d);
+    waves += __shfl_xor_sync(0xffffffffu, waves, d);
+  }
   if (lane == 0) {
+    // hash accumulator candidate (reading R31): its waves (one entry x <= 32 entries of
+    // the entry's B row) keep at least half of the lanes busy; short B rows stay in
+    // AC-ESC, whose draws pack them densely
+    if (hash_ok) hash_ok[b] = sum > 0 && 2 * sum >= 32 * waves;
     products[b] = sum;
-    slots[b] = (sum + (CAP - KEEP) - 1) / (CAP - KEEP);
+    // the hash accumulator (R31) emits up to one chunk per warp
+    slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)HASH_WARPS) : 0;
     nz_begin[b] = (int32_t)nzb;
     nz_end[b] = (int32_t)nze;
   }
@@ -137,11 +151,11 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
 
 void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* nzb, int32_t* nze,
-                         int64_t* products, int64_t* slots, cudaStream_t st) {
+                         int64_t* products, int64_t* slots, int32_t* hash_ok, cudaStream_t st) {
   if (max_blocks == 0) return;
   const int T = 256, WPB = T / 32;
   k_block_bounds<<<(unsigned)((max_blocks + WPB - 1) / WPB), T, 0, st>>>(
-      A.row_ptr, A.col, B.row_ptr, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots);
+      A.row_ptr, A.col, B.row_ptr, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots, hash_ok);
 }
 
 // Canonical-CSR check (reading R3): row_ptr monotone, columns strictly increasing and

@@ -22,7 +22,8 @@ void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* block_r
                 int64_t max_blocks, cudaStream_t st);
 void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* blk_nz_begin,
-                         int32_t* blk_nz_end, int64_t* blk_products, int64_t* blk_slots, cudaStream_t st);
+                         int32_t* blk_nz_end, int64_t* blk_products, int64_t* blk_slots,
+                         int32_t* blk_hash_ok /* nullable: hash-accumulator candidates (R31) */, cudaStream_t st);
 
 // ---- device-wide exclusive scan (scan.cu) --------------------------------------
 // out[i] = sum_{j<i} in[j] for i < n, total -> *total_dev.  tmp needs scan_tmp_elems(n).
@@ -48,8 +49,13 @@ struct EscArgs {
   int32_t* nchunks;             // per block
   int32_t* used;                // per block: chunk elements written
   int32_t* row_count;           // per row of C
+  int32_t* hash_done;           // per block: in: 1 = hash candidate (k_block_bounds); out: 1 = finished
+                                // by k_hash, AC-ESC skips it (nullptr: none)
+  int64_t* hash_count;          // blocks finished by k_hash (atomic counter, info only)
 };
 void launch_esc(const EscArgs& a, bool f64, cudaStream_t st);
+// adaptive alternative (hash.cu, reading R31): must run before launch_esc on the same stream
+void launch_hash(const EscArgs& a, bool f64, cudaStream_t st);
 
 // ---- stage 3: chunk ordering, shared rows, merges (merge.cu) --------------------
 struct MergeState {

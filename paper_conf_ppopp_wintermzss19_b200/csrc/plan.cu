@@ -60,7 +60,8 @@ struct DevBuf {
 constexpr int H_SEG_ROWS = 32;
 constexpr int H_SEG_INFO = H_SEG_ROWS + MAX_SEGMENTS + 1;
 constexpr int H_SCAL_WORDS = H_SEG_INFO + MAX_SEGMENTS + 1;
-enum Stage { S_GLB = 0, S_ESC, S_MCC, S_MM, S_PM, S_SM, S_SCAN, S_CC, S_END, NSTAGE_EV };
+// S_HASHEND: end of the hash-accumulator part of the ESC stage (stage 8 "HASH")
+enum Stage { S_GLB = 0, S_ESC, S_MCC, S_MM, S_PM, S_SM, S_SCAN, S_CC, S_END, S_HASHEND, NSTAGE_EV };
 
 }  // namespace
 
@@ -72,7 +73,7 @@ struct acspgemm_plan_s {
   DevBuf seg, seg_rows, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base;
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
-  DevBuf cur_first, cur_last, err, bused, bused_scan;
+  DevBuf cur_first, cur_last, err, bused, bused_scan, hdone;
   DevBuf lgiant, g_lo, g_nsl, g_base, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30): lists, spans, slices
   // acspgemm_multiply_host: device copies of A and B, two C piece buffers, copy stream
   DevBuf hp_a[3], hp_b[3], hp_c[2][3];
@@ -151,7 +152,7 @@ int64_t helper_bytes(acspgemm_plan p) {
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->descs, &p->dense, &p->sflag,
                   &p->spos, &p->shared, &p->row_count, &p->row_ptr, &p->scan_tmp, &p->kflag, &p->kpos,
                   &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
-                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan};
+                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->hdone};
   int64_t t = 0;
   for (DevBuf* b : bs) t += (int64_t)b->bytes;
   return t;
@@ -243,6 +244,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->chunk_base, sizeof(int64_t) * max_blocks);
   ACS_ENSURE(p->bused, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->bused_scan, sizeof(int64_t) * max_blocks);
+  ACS_ENSURE(p->hdone, sizeof(int32_t) * max_blocks);
   const int64_t tmp_n = scan_tmp_elems(std::max<int64_t>(max_blocks, A->rows) * 2 + 1024);
   ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * tmp_n);
   int32_t* nblocks_dev = reinterpret_cast<int32_t*>(scal + 20);
@@ -251,7 +253,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   launch_glb(Av, nseg, ptr<int64_t>(p->seg), ptr<int32_t>(p->brs), max_blocks, st);
   tl_launches += 1;
   launch_block_bounds(Av, Bv, nseg, ptr<int64_t>(p->seg), nblocks_dev, max_blocks, ptr<int32_t>(p->nzb),
-                      ptr<int32_t>(p->nze), ptr<int64_t>(p->bprod), ptr<int64_t>(p->bslot), st);
+                      ptr<int32_t>(p->nze), ptr<int64_t>(p->bprod), ptr<int64_t>(p->bslot),
+                      p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE ? ptr<int32_t>(p->hdone) : nullptr, st);
   tl_launches += 1;
   launch_scan_i64(ptr<int64_t>(p->bprod), ptr<int64_t>(p->pool_off), max_blocks, scal + 0, ptr<int64_t>(p->scan_tmp), st);
   launch_scan_i64(ptr<int64_t>(p->bslot), ptr<int64_t>(p->desc_off), max_blocks, scal + 1, ptr<int64_t>(p->scan_tmp), st);
@@ -298,6 +301,16 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.nchunks = ptr<int32_t>(p->nchunks);
   ea.used = ptr<int32_t>(p->bused);
   ea.row_count = ptr<int32_t>(p->row_count);
+  ea.hash_done = nullptr;
+  ea.hash_count = scal + 6;
+  ACS_CUDA(cudaMemsetAsync(scal + 6, 0, sizeof(int64_t), st));
+  if (p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE) {
+    // hash accumulator first (reading R31); blocks it does not finish go to AC-ESC
+    ea.hash_done = ptr<int32_t>(p->hdone);
+    launch_hash(ea, p->f64, st);
+    tl_launches += nblocks > 0 ? 1 : 0;
+  }
+  record(p, S_HASHEND, st);
   launch_esc(ea, p->f64, st);
   tl_launches += nblocks > 0 ? 1 : 0;
   ACS_CUDA(cudaGetLastError());
@@ -329,7 +342,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   launch_find_shared(ms, scal + 4, st);
   tl_launches += 1 + (slots > 0 ? 5 : 0);
   ACS_CUDA(cudaGetLastError());
-  if ((s = sync_read(p, scal + 3, 3, st)) != ACSPGEMM_OK) return s;
+  if ((s = sync_read(p, scal + 3, 4, st)) != ACSPGEMM_OK) return s;
+  p->info.nhash_blocks = p->h_scal[3];
   p->total_chunks = p->h_scal[0];
   p->nshared = p->h_scal[1];
   p->max_chunks = slots;
@@ -629,6 +643,7 @@ void acspgemm_options_default(acspgemm_options* opt) {
   opt->validate_inputs = 0;
   opt->collect_stage_times = 0;
   opt->num_segments = DEFAULT_SEGMENTS;
+  opt->strategy = ACSPGEMM_STRATEGY_ADAPTIVE;
 }
 
 acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options* opt) {
@@ -641,6 +656,10 @@ acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options
   if (p->opt.num_segments > MAX_SEGMENTS) {
     delete p;
     return set_err(ACSPGEMM_ERR_INVALID_ARG, "num_segments > 64");
+  }
+  if (p->opt.strategy != ACSPGEMM_STRATEGY_ADAPTIVE && p->opt.strategy != ACSPGEMM_STRATEGY_ESC) {
+    delete p;
+    return set_err(ACSPGEMM_ERR_INVALID_ARG, "unknown strategy");
   }
   std::memset(&p->info, 0, sizeof(p->info));
   // mapped: read-backs are written by a kernel (launch_read_back), not a copy engine
@@ -893,13 +912,15 @@ acspgemm_status acspgemm_stage_times(acspgemm_plan p, float* ms_out, int n) {
   if (!p || !ms_out) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
   if (!p->opt.collect_stage_times || !p->ev_ok) return set_err(ACSPGEMM_ERR_NOT_READY, "stage times not collected");
   if (p->empty) {
-    for (int i = 0; i < n && i < 8; ++i) ms_out[i] = 0.f;
+    for (int i = 0; i < n && i < 9; ++i) ms_out[i] = 0.f;
     return ACSPGEMM_OK;
   }
   ACS_CUDA(cudaEventSynchronize(p->ev[S_END]));
-  for (int i = 0; i < n && i < 8; ++i) {
+  for (int i = 0; i < n && i < 9; ++i) {
     float ms = 0.f;
-    if (cudaEventElapsedTime(&ms, p->ev[i], p->ev[i + 1]) != cudaSuccess) { cudaGetLastError(); ms = -1.f; }
+    // stage 8 (HASH) is the hash-accumulator part of stage 1 (ESC)
+    const int a = i < 8 ? i : (int)S_ESC, b = i < 8 ? i + 1 : (int)S_HASHEND;
+    if (cudaEventElapsedTime(&ms, p->ev[a], p->ev[b]) != cudaSuccess) { cudaGetLastError(); ms = -1.f; }
     ms_out[i] = ms;
   }
   return ACSPGEMM_OK;

@@ -16,7 +16,7 @@ def run(name, A, B, dt, reps=5):
     info = plan.info(); st = plan.stage_times()
     out = {"workload": name, "dtype": str(np.dtype(dt)), "ms_per_multiply": ms, "GFLOPS": 2 * info["products"] / (ms * 1e-3) / 1e9,
            "products": info["products"], "nnz_c": info["nnz_c"], "stages_ms": {k: round(v, 3) for k, v in st.items()},
-           "nshared": info["nshared"], "nmulti": info["nmulti"], "npath": info["npath"], "nsearch": info["nsearch"]}
+           "nshared": info["nshared"], "nmulti": info["nmulti"], "npath": info["npath"], "nsearch": info["nsearch"], "nhash": info["nhash_blocks"], "nblocks": info["nblocks"]}
     print(json.dumps(out), flush=True)
     plan.close(); del dA, dB; torch.cuda.empty_cache()
 CFGS = sys.argv[1].split(",") if len(sys.argv) > 1 else ["cfg1", "cfg2", "cfg3", "cfg5", "cfg4"]

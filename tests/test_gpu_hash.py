@@ -1,0 +1,188 @@
+"""GPU parity of the adaptive strategy (reading R31): the hash accumulator that blocks
+try before AC-ESC (§5), against the CPU oracle and
+against the ESC-only strategy, through the C ABI.
+
+What pins it:
+  * rows that lie inside one block are summed left to right in A-entry order, the order
+    of the oracle's Gustavson accumulator (oracle/gustavson.c: t = a*b; acc += t), so
+    fp64 values are bit-identical to the oracle's there (random U(-1,1) values);
+  * structure bit-exact, values within the north-star tolerance everywhere;
+  * products of one column inside a 32-product wave (short B rows sharing columns),
+    empty B rows (more than a warp of them in a row), rows with more distinct columns
+    than the table holds (fallback to AC-ESC) and mixed blocks;
+  * bit-identical results run to run and across canonical-segment splits.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from oracle import alg
+from synth import from_coo, poisson2d_5pt, poisson3d_27pt, power_law_csr, random_csr, random_rowlen_csr, rmat
+
+from test_gpu_parity import TOL, assert_parity, digest, gpu_mult, pkg
+
+pytestmark = pytest.mark.gpu
+
+
+def run(A, B, dt, strategy="adaptive"):
+    p = pkg()
+    plan = p.Plan(strategy=strategy)
+    dA = p.DeviceCSR.from_host(A, "cuda", dt)
+    dB = p.DeviceCSR.from_host(B, "cuda", dt)
+    C = plan.multiply(dA, dB)
+    torch.cuda.synchronize()
+    out = C.to_numpy()
+    info = plan.info()
+    plan.close()
+    return out, info
+
+
+def check(out, A, B, dt):
+    rp, col, val = out
+    ref = oracle.gustavson(A.astype(dt), B.astype(dt))
+    assert (rp == ref.row_ptr).all() and (col == ref.col).all()
+    err = np.abs(val.astype(np.float64) - ref.val)
+    assert not (err > TOL[dt] * ref.absval).any()
+    return ref
+
+
+def test_hash_left_fold_bit_exact_fp64(cuda_available):
+    """Rows of 8 entries never straddle a 512-entry block: every row is finished by
+    one warp, and its fp64 sums equal the oracle's left fold bit for bit."""
+    n = 4096
+    A = random_rowlen_csr(n, n, np.full(n, 8), seed=11)
+    B = random_rowlen_csr(n, n, np.random.default_rng(12).integers(16, 32, n), seed=12)
+    out, info = run(A, B, np.float64)
+    ref = check(out, A, B, np.float64)
+    assert info["nhash_blocks"] == info["nblocks"]
+    assert (out[2] == ref.val).all(), "hash accumulator is not the left fold in A-entry order"
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_hash_shared_columns_across_waves(dt, cuda_available):
+    """B rows drawn from few columns (and longer than a warp): every column collects
+    products from many waves, added in expansion order (bit-exact left fold on rows
+    inside one block)."""
+    n = 600
+    rng = np.random.default_rng(5)
+    B = random_rowlen_csr(n, 70, rng.integers(16, 60, n), seed=7)
+    A = random_rowlen_csr(300, n, rng.integers(1, 30, 300), seed=6)
+    out, info = run(A, B, dt)
+    ref = check(out, A, B, dt)
+    assert info["nhash_blocks"] == info["nblocks"]
+    if dt == np.float64:
+        # rows inside one block are bit-exact (left fold); blocks of 512 nonzeros are
+        # counted from each canonical segment's first nonzero (reading R21)
+        rp = A.row_ptr.astype(np.int64)
+        seg = alg.canonical_segments(A.row_ptr, 8)
+        s_of = np.searchsorted(np.asarray(seg[1:]), np.arange(A.rows), side="right")
+        base = rp[np.asarray(seg)[s_of]]
+        inside = ((rp[:-1] - base) // 512) == ((rp[1:] - 1 - base) // 512)
+        crp = ref.row_ptr.astype(np.int64)
+        assert inside.sum() > 200
+        for i in np.nonzero(inside)[0]:
+            s, e = crp[i], crp[i + 1]
+            assert (out[2][s:e] == ref.val[s:e]).all()
+
+
+def test_hash_empty_b_rows(cuda_available):
+    """Entries whose B rows are empty add no waves, including runs of them and empty
+    first/last entries of a row, and rows whose B rows are all empty."""
+    n = 2000
+    rng = np.random.default_rng(8)
+    blen = rng.integers(16, 32, n)
+    blen[rng.random(n) < 0.6] = 0
+    blen[100:200] = 0                       # long run of empty B rows
+    B = random_rowlen_csr(n, 5000, blen, seed=9)
+    r, c = [], []
+    for i in range(400):
+        k = rng.choice(n, size=int(rng.integers(1, 16)), replace=False)
+        if i % 3 == 0:
+            k = np.concatenate([k, np.arange(100, 160)])   # > 32 consecutive empty entries
+        if i % 7 == 0:
+            k = np.arange(120, 140)                          # only empty B rows
+        k = np.unique(k)
+        r += [i] * len(k)
+        c += k.tolist()
+    A = from_coo(400, n, np.array(r), np.array(c), rng.uniform(-1, 1, len(r)))
+    out, info = run(A, B, np.float64)
+    check(out, A, B, np.float64)
+    assert info["nhash_blocks"] == info["nblocks"]
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_short_b_rows_stay_in_esc(dt, cuda_available):
+    """Blocks whose waves would leave most lanes idle (B rows of 1..8 entries) are not
+    hash candidates: AC-ESC computes them."""
+    rng = np.random.default_rng(2)
+    A = random_rowlen_csr(2000, 3000, rng.integers(1, 40, 2000), seed=3)
+    B = random_rowlen_csr(3000, 2500, rng.integers(1, 9, 3000), seed=4)
+    out, info = run(A, B, dt)
+    check(out, A, B, dt)
+    assert info["nhash_blocks"] == 0
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_hash_overflow_falls_back_to_esc(dt, cuda_available):
+    """Rows with more than HASH_UMAX = 256 distinct columns send their block to AC-ESC;
+    blocks without such rows stay in the hash accumulator; the result is the same C."""
+    n = 20000
+    rng = np.random.default_rng(3)
+    lens = rng.integers(1, 8, 3000)
+    lens[1500:1530] = 40                    # 40 x ~24 products, ~950 distinct columns
+    A = random_rowlen_csr(3000, n, lens, seed=4)
+    B = random_rowlen_csr(n, n, rng.integers(17, 32, n), seed=5)
+    out, info = run(A, B, dt)
+    check(out, A, B, dt)
+    assert 0 < info["nhash_blocks"] < info["nblocks"]
+    esc, info_e = run(A, B, dt, strategy="esc")
+    check(esc, A, B, dt)
+    assert info_e["nhash_blocks"] == 0
+    assert (esc[0] == out[0]).all() and (esc[1] == out[1]).all()
+
+
+@pytest.mark.parametrize("strategy", ["adaptive", "esc"])
+@pytest.mark.parametrize("case", ["poisson2d", "poisson27", "rmat", "powerlaw", "random"])
+def test_strategies_parity(strategy, case, cuda_available):
+    if case == "poisson2d":
+        A = B = poisson2d_5pt(64); exact = True
+    elif case == "poisson27":
+        A = B = poisson3d_27pt(14); exact = True
+    elif case == "rmat":
+        A = B = rmat(scale=12, edge_factor=16, values="uniform"); exact = False
+    elif case == "powerlaw":
+        A = B = power_law_csr(3000, 3000, mean_len=12, alpha=1.4, max_len=900, seed=21); exact = False
+    else:
+        A = random_csr(2500, 1800, 0.01, seed=31); B = random_csr(1800, 2200, 0.01, seed=32); exact = False
+    for dt in (np.float64, np.float32):
+        assert_parity(A, B, dt, exact=exact and dt == np.float64, strategy=strategy)
+
+
+def test_hash_bit_stable_runs_and_splits(cuda_available):
+    """The adaptive strategy is bit-identical run to run and for every segment count."""
+    p = pkg()
+    A = poisson3d_27pt(20)
+    A.val[:] = np.random.default_rng(1).uniform(-1, 1, A.val.shape)
+    hs = set()
+    for nseg in (1, 2, 8, 8, 37):
+        plan = p.Plan(num_segments=nseg)
+        dA = p.DeviceCSR.from_host(A, "cuda", np.float64)
+        C = plan.multiply(dA, dA)
+        torch.cuda.synchronize()
+        if nseg == 8:
+            hs.add(digest(*C.to_numpy()))
+        assert plan.info()["nhash_blocks"] == plan.info()["nblocks"]
+        check(C.to_numpy(), A, A, np.float64)
+        plan.close()
+    assert len(hs) == 1
+
+
+def test_hash_stencil_square_exact(cuda_available):
+    """27-point stencil squared (integer values): every block is finished by the hash
+    accumulator and the result is exact."""
+    A = poisson3d_27pt(24)
+    out, info = run(A, A, np.float64)
+    ref = check(out, A, A, np.float64)
+    assert info["nhash_blocks"] == info["nblocks"]
+    assert (out[2] == ref.val).all()
