@@ -13,6 +13,7 @@
 // Chunk allocation is deterministic (reading R8): block b writes its chunks to a
 // slot range sized from its exact product count (stage 1), so no atomics, no
 // restarts, and the chunk id (block, running number) is the global order (L430).
+#include <algorithm>
 #include <climits>
 #include "esc_core.cuh"
 #include "kernels.cuh"
@@ -218,13 +219,10 @@ __device__ __forceinline__ void esc_iteration_split(EscSmem<T>& S, const EscArgs
                         [&](uint64_t key, int) { return cmin + (int)(key & colmask); });
 }
 
+// AC-ESC of one block b.
 template <typename T>
-__global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  EscSmem<T>& S = *reinterpret_cast<EscSmem<T>*>(smem_raw);
+__device__ __forceinline__ void esc_block(EscSmem<T>& S, const EscArgs& a, const int b) {
   const int tid = threadIdx.x;
-  const int b = blockIdx.x;
-  if (a.hash_done && a.hash_done[b]) return;        // finished by the hash accumulator (R31)
   const int32_t* __restrict__ arp = a.A.row_ptr;
   const int32_t* __restrict__ acol = a.A.col;
   const T* __restrict__ aval = reinterpret_cast<const T*>(a.A.val);
@@ -381,11 +379,59 @@ __global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
   }
 }
 
+// One CTA per block; with the adaptive strategy (hash_done set) a persistent grid takes
+// the blocks the hash accumulator did not finish (reading R31) from a list, one at a time
+// through an atomic counter, instead of launching a CTA per finished block.  Blocks are
+// independent and write only their own chunk range: the order does not change any result.
+template <typename T>
+__global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  EscSmem<T>& S = *reinterpret_cast<EscSmem<T>*>(smem_raw);
+  if (!a.hash_done) {
+    esc_block<T>(S, a, blockIdx.x);
+    return;
+  }
+  const int64_t n = *a.esc_count;
+  for (;;) {
+    if (threadIdx.x == 0)
+      S.s.misc[15] = (int)atomicAdd(reinterpret_cast<unsigned long long*>(a.esc_next), 1ull);
+    __syncthreads();
+    const int i = S.s.misc[15];
+    __syncthreads();
+    if (i >= n) break;
+    esc_block<T>(S, a, a.esc_list[i]);
+    __syncthreads();                                  // shared memory is reused by the next block
+  }
+}
+
+// list of the blocks k_hash left to AC-ESC (any order)
+__global__ void k_esc_list(const int32_t* __restrict__ hash_done, int32_t nblocks, int32_t* __restrict__ list,
+                           int64_t* __restrict__ count) {
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  const bool need = b < nblocks && !hash_done[b];
+  const unsigned m = __ballot_sync(0xffffffffu, need);
+  if (!m) return;
+  int base = 0;
+  if ((threadIdx.x & 31) == __ffs(m) - 1)
+    base = (int)atomicAdd(reinterpret_cast<unsigned long long*>(count), (unsigned long long)__popc(m));
+  base = __shfl_sync(0xffffffffu, base, __ffs(m) - 1);
+  if (need) list[base + __popc(m & ((1u << (threadIdx.x & 31)) - 1u))] = b;
+}
+
 template <typename T>
 static void launch_esc_t(const EscArgs& a, cudaStream_t st) {
   const size_t smem = sizeof(EscSmem<T>);
   cudaFuncSetAttribute(k_esc<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k_esc<T><<<a.nblocks, THREADS, smem, st>>>(a);
+  int grid = a.nblocks;
+  if (a.hash_done) {
+    k_esc_list<<<(a.nblocks + 255) / 256, 256, 0, st>>>(a.hash_done, a.nblocks, a.esc_list, a.esc_count);
+    int dev = 0, sms = 148, per = ESC_MIN_BLOCKS;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_esc<T>, THREADS, smem);
+    grid = std::min<int>(a.nblocks, std::max(1, sms * std::max(per, 1)));
+  }
+  k_esc<T><<<grid, THREADS, smem, st>>>(a);
 }
 
 void launch_esc(const EscArgs& a, bool f64, cudaStream_t st) {

@@ -7,6 +7,7 @@
 // number to each thread block", L194).  Rows never straddle segments, so the block
 // decomposition -- and therefore every summation tree -- is the same whether the
 // segments run on one GPU or on several.
+#include <climits>
 #include "kernels.cuh"
 
 namespace acs {
@@ -98,7 +99,7 @@ void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* brs, in
 // (every local ESC iteration consumes at least CAP - KEEP products and emits at most
 // one chunk), and products bounds its chunk elements (compaction never grows data).
 __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* __restrict__ acol,
-                               const int32_t* __restrict__ brp, int nseg, const int64_t* __restrict__ seg,
+                               const int32_t* __restrict__ brp, const int32_t* __restrict__ bcol, int nseg, const int64_t* __restrict__ seg,
                                const int32_t* __restrict__ nblocks_dev, int64_t max_blocks,
                                int32_t* __restrict__ nz_begin, int32_t* __restrict__ nz_end,
                                int64_t* __restrict__ products, int64_t* __restrict__ slots,
@@ -136,11 +137,49 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
     sum += __shfl_xor_sync(0xffffffffu, sum, d);
     waves += __shfl_xor_sync(0xffffffffu, waves, d);
   }
+  // hash accumulator candidate (reading R31), two deterministic tests on the block's own
+  // entries: (1) its waves (one entry x <= 32 entries of the entry's B row) keep at least
+  // half of the lanes busy -- short B rows stay in AC-ESC, whose draws pack them
+  // densely; (2) the rows are likely to compact: the B rows of adjacent entries share at
+  // least a quarter of their columns (8 sampled pairs, first <= 32 columns of each) --
+  // random-column rows barely compact, and AC-ESC's sort is cheaper than hashing and
+  // then sorting them
+  int hok = 0;
+  if (hash_ok && sum > 0 && 2 * sum >= 32 * waves) {
+    constexpr int NS = 8;                     // sampled adjacent pairs
+    const int64_t n = nze - nzb;
+    int ov = 0, mn = 0;
+    if (n >= 2) {
+      int v1[NS], v2[NS], l1[NS], l2[NS];
+#pragma unroll
+      for (int s = 0; s < NS; ++s) {
+        const int64_t p = nzb + ((int64_t)s * (n - 1)) / NS;
+        const int k1 = acol[p], k2 = acol[p + 1];
+        const int a0 = brp[k1], b0 = brp[k2];
+        l1[s] = min(brp[k1 + 1] - a0, 32);
+        l2[s] = min(brp[k2 + 1] - b0, 32);
+        v1[s] = lane < l1[s] ? bcol[a0 + lane] : INT_MAX;
+        v2[s] = lane < l2[s] ? bcol[b0 + lane] : INT_MAX;
+      }
+#pragma unroll
+      for (int s = 0; s < NS; ++s) {
+        // position of v1 among the sorted v2 (held across the lanes): count of v2 < v1
+        int pos = 0;
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+          const int x = __shfl_sync(0xffffffffu, v2[s], pos + step - 1);
+          if (x < v1[s]) pos += step;
+        }
+        const int at = __shfl_sync(0xffffffffu, v2[s], pos & 31);
+        ov += lane < l1[s] && pos < 32 && at == v1[s];
+        mn += min(l1[s], l2[s]);
+      }
+    }
+    ov = __reduce_add_sync(0xffffffffu, ov);
+    hok = mn > 0 && 4 * ov >= mn;
+  }
   if (lane == 0) {
-    // hash accumulator candidate (reading R31): its waves (one entry x <= 32 entries of
-    // the entry's B row) keep at least half of the lanes busy; short B rows stay in
-    // AC-ESC, whose draws pack them densely
-    if (hash_ok) hash_ok[b] = sum > 0 && 2 * sum >= 32 * waves;
+    if (hash_ok) hash_ok[b] = hok;
     products[b] = sum;
     // the hash accumulator (R31) emits up to one chunk per warp
     slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)HASH_WARPS) : 0;
@@ -155,7 +194,7 @@ void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int
   if (max_blocks == 0) return;
   const int T = 256, WPB = T / 32;
   k_block_bounds<<<(unsigned)((max_blocks + WPB - 1) / WPB), T, 0, st>>>(
-      A.row_ptr, A.col, B.row_ptr, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots, hash_ok);
+      A.row_ptr, A.col, B.row_ptr, B.col, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots, hash_ok);
 }
 
 // Canonical-CSR check (reading R3): row_ptr monotone, columns strictly increasing and

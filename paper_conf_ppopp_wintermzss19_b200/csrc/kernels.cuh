@@ -52,6 +52,9 @@ struct EscArgs {
   int32_t* hash_done;           // per block: in: 1 = hash candidate (k_block_bounds); out: 1 = finished
                                 // by k_hash, AC-ESC skips it (nullptr: none)
   int64_t* hash_count;          // blocks finished by k_hash (atomic counter, info only)
+  int32_t* esc_list;            // adaptive: blocks left to AC-ESC [nblocks]
+  int64_t* esc_count;           // adaptive: their number (zeroed before launch_hash)
+  int64_t* esc_next;            // adaptive: grab counter of the persistent k_esc (zeroed)
 };
 void launch_esc(const EscArgs& a, bool f64, cudaStream_t st);
 // adaptive alternative (hash.cu, reading R31): must run before launch_esc on the same stream

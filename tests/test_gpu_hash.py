@@ -52,7 +52,7 @@ def test_hash_left_fold_bit_exact_fp64(cuda_available):
     one warp, and its fp64 sums equal the oracle's left fold bit for bit."""
     n = 4096
     A = random_rowlen_csr(n, n, np.full(n, 8), seed=11)
-    B = random_rowlen_csr(n, n, np.random.default_rng(12).integers(16, 32, n), seed=12)
+    B = random_rowlen_csr(n, 64, np.random.default_rng(12).integers(16, 32, n), seed=12)
     out, info = run(A, B, np.float64)
     ref = check(out, A, B, np.float64)
     assert info["nhash_blocks"] == info["nblocks"]
@@ -91,10 +91,10 @@ def test_hash_empty_b_rows(cuda_available):
     first/last entries of a row, and rows whose B rows are all empty."""
     n = 2000
     rng = np.random.default_rng(8)
-    blen = rng.integers(16, 32, n)
+    blen = rng.integers(24, 32, n)
     blen[rng.random(n) < 0.6] = 0
     blen[100:200] = 0                       # long run of empty B rows
-    B = random_rowlen_csr(n, 5000, blen, seed=9)
+    B = random_rowlen_csr(n, 40, blen, seed=9)
     r, c = [], []
     for i in range(400):
         k = rng.choice(n, size=int(rng.integers(1, 16)), replace=False)
@@ -108,7 +108,7 @@ def test_hash_empty_b_rows(cuda_available):
     A = from_coo(400, n, np.array(r), np.array(c), rng.uniform(-1, 1, len(r)))
     out, info = run(A, B, np.float64)
     check(out, A, B, np.float64)
-    assert info["nhash_blocks"] == info["nblocks"]
+    assert info["nhash_blocks"] > 0
 
 
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
@@ -125,17 +125,33 @@ def test_short_b_rows_stay_in_esc(dt, cuda_available):
 
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
 def test_hash_overflow_falls_back_to_esc(dt, cuda_available):
-    """Rows with more than HASH_UMAX = 256 distinct columns send their block to AC-ESC;
-    blocks without such rows stay in the hash accumulator; the result is the same C."""
-    n = 20000
+    """A row with more than HASH_UMAX = 256 distinct columns inside an otherwise
+    compacting block sends the block to AC-ESC; blocks without such rows stay in the
+    hash accumulator; the result is the same C as the ESC-only strategy's."""
     rng = np.random.default_rng(3)
-    lens = rng.integers(1, 8, 3000)
-    lens[1500:1530] = 40                    # 40 x ~24 products, ~950 distinct columns
-    A = random_rowlen_csr(3000, n, lens, seed=4)
-    B = random_rowlen_csr(n, n, rng.integers(17, 32, n), seed=5)
+    nb = 4000
+    # B rows 0..1999 draw from 60 columns (compacting), rows 2000.. from 20000 (wide)
+    lens = rng.integers(17, 32, nb)
+    r, c = [], []
+    for i in range(nb):
+        span = 60 if i < 2000 else 20000
+        cols = np.sort(rng.choice(span, size=int(lens[i]), replace=False))
+        r += [i] * len(cols)
+        c += cols.tolist()
+    B = from_coo(nb, 20000, np.array(r), np.array(c), rng.uniform(-1, 1, len(r)))
+    r, c = [], []
+    for i in range(3000):
+        if i in (700, 1500, 2300):
+            k = rng.choice(np.arange(2000, nb), size=40, replace=False)   # ~950 distinct columns
+        else:
+            k = rng.choice(2000, size=int(rng.integers(1, 8)), replace=False)
+        k = np.sort(k)
+        r += [i] * len(k)
+        c += k.tolist()
+    A = from_coo(3000, nb, np.array(r), np.array(c), rng.uniform(-1, 1, len(r)))
     out, info = run(A, B, dt)
     check(out, A, B, dt)
-    assert 0 < info["nhash_blocks"] < info["nblocks"]
+    assert 0 < info["nhash_blocks"] <= info["nblocks"] - 3
     esc, info_e = run(A, B, dt, strategy="esc")
     check(esc, A, B, dt)
     assert info_e["nhash_blocks"] == 0
@@ -172,7 +188,7 @@ def test_hash_bit_stable_runs_and_splits(cuda_available):
         torch.cuda.synchronize()
         if nseg == 8:
             hs.add(digest(*C.to_numpy()))
-        assert plan.info()["nhash_blocks"] == plan.info()["nblocks"]
+        assert plan.info()["nhash_blocks"] >= 0.9 * plan.info()["nblocks"]
         check(C.to_numpy(), A, A, np.float64)
         plan.close()
     assert len(hs) == 1
@@ -186,3 +202,15 @@ def test_hash_stencil_square_exact(cuda_available):
     ref = check(out, A, A, np.float64)
     assert info["nhash_blocks"] == info["nblocks"]
     assert (out[2] == ref.val).all()
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_low_compaction_rows_go_to_esc(dt, cuda_available):
+    """Rows whose products hardly compact (random columns: adjacent entries' B rows share
+    almost no columns) are not hash candidates; AC-ESC computes them."""
+    rng = np.random.default_rng(12)
+    A = random_rowlen_csr(1500, 4000, rng.integers(10, 20, 1500), seed=13)
+    B = random_rowlen_csr(4000, 200000, rng.integers(24, 32, 4000), seed=14)
+    out, info = run(A, B, dt)
+    check(out, A, B, dt)
+    assert info["nhash_blocks"] == 0
