@@ -12,20 +12,30 @@
 
 namespace acs {
 
-// One warp per chunk (or shared row): 4 independent element loads per lane in flight.
+// One warp per chunk (or shared row): 8 independent element loads per lane in flight
+// (the copy is bound by DRAM latency x bytes in flight, not by instructions).
 template <typename T>
 __device__ __forceinline__ void warp_copy(const int32_t* __restrict__ scol, const T* __restrict__ sval,
                                           int32_t* __restrict__ dcol, T* __restrict__ dval, int n, int lane) {
+  constexpr int U = 8;
   int i = lane;
-  for (; i + 96 < n; i += 128) {
-    const int32_t c0 = __ldcs(scol + i), c1 = __ldcs(scol + i + 32), c2 = __ldcs(scol + i + 64), c3 = __ldcs(scol + i + 96);
-    const T v0 = __ldcs(sval + i), v1 = __ldcs(sval + i + 32), v2 = __ldcs(sval + i + 64), v3 = __ldcs(sval + i + 96);
-    __stcs(dcol + i, c0); __stcs(dcol + i + 32, c1); __stcs(dcol + i + 64, c2); __stcs(dcol + i + 96, c3);
-    __stcs(dval + i, v0); __stcs(dval + i + 32, v1); __stcs(dval + i + 64, v2); __stcs(dval + i + 96, v3);
+  for (; i + 32 * (U - 1) < n; i += 32 * U) {
+    int32_t c[U];
+    T v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) { c[u] = __ldcs(scol + i + 32 * u); v[u] = __ldcs(sval + i + 32 * u); }
+#pragma unroll
+    for (int u = 0; u < U; ++u) { __stcs(dcol + i + 32 * u, c[u]); __stcs(dval + i + 32 * u, v[u]); }
   }
-  for (; i < n; i += 32) {
-    __stcs(dcol + i, __ldcs(scol + i));
-    __stcs(dval + i, __ldcs(sval + i));
+  int32_t c[U];
+  T v[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    if (i + 32 * u < n) { c[u] = __ldcs(scol + i + 32 * u); v[u] = __ldcs(sval + i + 32 * u); }
+  }
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    if (i + 32 * u < n) { __stcs(dcol + i + 32 * u, c[u]); __stcs(dval + i + 32 * u, v[u]); }
   }
 }
 
