@@ -23,10 +23,14 @@ namespace acs {
 constexpr int THREADS = ACS_THREADS;         // threads per CTA (paper: 256, L344)
 constexpr int ITEMS = ACS_ITEMS;             // sorted elements per thread (paper: 8, L556)
 constexpr int CAP = THREADS * ITEMS;         // products per local ESC iteration (2048)
-constexpr int IDXBITS = 11;                  // log2(CAP): position bits in a sort word
+constexpr int IDXBITS = 31 - __builtin_clz(CAP); // log2(CAP): position bits in a sort word
 constexpr int NPB = 512;                     // NNZ_PER_BLOCK (Alg. 1, Alg. 2; L556 "256/512")
 constexpr int NNZ_PER_THREAD = NPB / THREADS;// A entries per thread
-constexpr int KEEP_PER_THREAD = 4;           // "keeps up to 4 elements per thread" (L556)
+#ifndef ACS_KEEP_PER_THREAD
+#define ACS_KEEP_PER_THREAD 4
+#endif
+constexpr int KEEP_PER_THREAD = ACS_KEEP_PER_THREAD; // "keeps up to 4 elements per thread" (L556)
+constexpr int CAP_SMALL = 512;               // small-tile AC-ESC (esc_small.cu, reading R32)
 constexpr int KEEP = KEEP_PER_THREAD * THREADS; // max kept elements of the last row
 #ifndef ACS_RADIX_BITS
 #define ACS_RADIX_BITS 5

@@ -55,8 +55,14 @@ struct EscArgs {
   int32_t* esc_list;            // adaptive: blocks left to AC-ESC [nblocks]
   int64_t* esc_count;           // adaptive: their number (zeroed before launch_hash)
   int64_t* esc_next;            // adaptive: grab counter of the persistent k_esc (zeroed)
+  const int64_t* blk_products;  // per block product count
+  int32_t* esc_list_small;      // adaptive: left blocks of <= CAP_SMALL products [nblocks]
+  int64_t* esc_count_small;     // (zeroed) -- the small-tile AC-ESC's list, counter
+  int64_t* esc_next_small;      // (zeroed)
 };
 void launch_esc(const EscArgs& a, bool f64, cudaStream_t st);
+// adaptive strategy: lists of the blocks k_hash left (big / small tile), before the ESCs
+void launch_esc_lists(const EscArgs& a, cudaStream_t st);
 // adaptive alternative (hash.cu, reading R31): must run before launch_esc on the same stream
 void launch_hash(const EscArgs& a, bool f64, cudaStream_t st);
 
@@ -161,3 +167,6 @@ void launch_add_offset(int32_t* p, int64_t n, int32_t off, cudaStream_t st);
 void launch_validate(const CsrView& M, int32_t* bad_flag, cudaStream_t st);
 
 }  // namespace acs
+
+// small-tile AC-ESC over esc_list_small (esc_small.cu, reading R32); args: acs::EscArgs
+void acs_launch_esc_small(const void* args, bool f64, cudaStream_t st);

@@ -73,7 +73,7 @@ struct acspgemm_plan_s {
   DevBuf seg, seg_rows, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base;
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
-  DevBuf cur_first, cur_last, err, bused, bused_scan, hdone, esc_list;
+  DevBuf cur_first, cur_last, err, bused, bused_scan, hdone, esc_list, esc_list_small;
   DevBuf lgiant, g_lo, g_nsl, g_base, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30): lists, spans, slices
   // acspgemm_multiply_host: device copies of A and B, two C piece buffers, copy stream
   DevBuf hp_a[3], hp_b[3], hp_c[2][3];
@@ -152,7 +152,7 @@ int64_t helper_bytes(acspgemm_plan p) {
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->descs, &p->dense, &p->sflag,
                   &p->spos, &p->shared, &p->row_count, &p->row_ptr, &p->scan_tmp, &p->kflag, &p->kpos,
                   &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
-                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->hdone, &p->esc_list};
+                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->hdone, &p->esc_list, &p->esc_list_small};
   int64_t t = 0;
   for (DevBuf* b : bs) t += (int64_t)b->bytes;
   return t;
@@ -246,6 +246,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->bused_scan, sizeof(int64_t) * max_blocks);
   ACS_ENSURE(p->hdone, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->esc_list, sizeof(int32_t) * max_blocks);
+  ACS_ENSURE(p->esc_list_small, sizeof(int32_t) * max_blocks);
   const int64_t tmp_n = scan_tmp_elems(std::max<int64_t>(max_blocks, A->rows) * 2 + 1024);
   ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * tmp_n);
   int32_t* nblocks_dev = reinterpret_cast<int32_t*>(scal + 20);
@@ -309,13 +310,25 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.esc_next = scal + 29;
   ACS_CUDA(cudaMemsetAsync(scal + 6, 0, sizeof(int64_t), st));
   ACS_CUDA(cudaMemsetAsync(scal + 28, 0, 2 * sizeof(int64_t), st));
+  ea.blk_products = ptr<int64_t>(p->bprod);
+  ea.esc_list_small = nullptr;
+  ea.esc_count_small = scal + 30;
+  ea.esc_next_small = scal + 31;
   if (p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE) {
-    // hash accumulator first (reading R31); blocks it does not finish go to AC-ESC
+    // hash accumulator first (reading R31); blocks it does not finish go to AC-ESC,
+    // small ones (<= 512 products) to the small-tile AC-ESC (reading R32)
+    ACS_CUDA(cudaMemsetAsync(scal + 30, 0, 2 * sizeof(int64_t), st));
     ea.hash_done = ptr<int32_t>(p->hdone);
+    ea.esc_list_small = ptr<int32_t>(p->esc_list_small);
     launch_hash(ea, p->f64, st);
     tl_launches += nblocks > 0 ? 1 : 0;
   }
   record(p, S_HASHEND, st);
+  if (ea.hash_done) {
+    launch_esc_lists(ea, st);
+    acs_launch_esc_small(&ea, p->f64, st);
+    tl_launches += nblocks > 0 ? 2 : 0;
+  }
   launch_esc(ea, p->f64, st);
   tl_launches += nblocks > 0 ? 1 : 0;
   ACS_CUDA(cudaGetLastError());

@@ -214,3 +214,27 @@ def test_low_compaction_rows_go_to_esc(dt, cuda_available):
     out, info = run(A, B, dt)
     check(out, A, B, dt)
     assert info["nhash_blocks"] == 0
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_small_tile_esc_blocks(dt, cuda_available):
+    """Blocks of <= 512 products that are not hash candidates run the small-tile AC-ESC
+    (reading R32), the others the default tile: A·P of a 7-point stencil and an
+    aggregation prolongator (exact, one product per A entry) next to denser rows."""
+    from synth import aggregation_prolongator, poisson3d_7pt
+    A = poisson3d_7pt(16)
+    P = aggregation_prolongator(16)
+    out, info = run(A, P, dt)
+    ref = check(out, A, P, dt)
+    assert info["nhash_blocks"] == 0
+    assert (out[2].astype(np.float64) == ref.val).all()
+    # mixed: short random rows (small blocks) and long ones (default tile)
+    rng = np.random.default_rng(21)
+    lens = np.where(rng.random(3000) < 0.5, 1, rng.integers(30, 120, 3000))
+    lens[:1200] = 1
+    A2 = random_rowlen_csr(3000, 2500, lens, seed=22)
+    B2 = random_rowlen_csr(2500, 2600, rng.integers(1, 6, 2500), seed=23)
+    out2, info2 = run(A2, B2, dt)
+    check(out2, A2, B2, dt)
+    esc2, _ = run(A2, B2, dt, strategy="esc")
+    assert (esc2[0] == out2[0]).all() and (esc2[1] == out2[1]).all()
