@@ -98,103 +98,110 @@ void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* brs, in
 // slots = ceil(products / (CAP - KEEP)) bounds the number of chunks the block emits
 // (every local ESC iteration consumes at least CAP - KEEP products and emits at most
 // one chunk), and products bounds its chunk elements (compaction never grows data).
+//
+// Hash accumulator candidate (reading R31), two deterministic tests on the block's own
+// entries: (1) its waves (one entry x <= 32 entries of the entry's B row) keep at least
+// half of the lanes busy -- short B rows stay in AC-ESC, whose draws pack them densely;
+// (2) the rows are likely to compact: the B rows of adjacent entries share at least a
+// quarter of their columns (8 sampled pairs, first <= 32 columns of each) -- random-
+// column rows barely compact, and AC-ESC's sort is cheaper than hashing and then
+// sorting them.  The candidates are counted (ncand) so that no k_hash is launched when
+// there is none.
 __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* __restrict__ acol,
-                               const int32_t* __restrict__ brp, const int32_t* __restrict__ bcol, int nseg, const int64_t* __restrict__ seg,
-                               const int32_t* __restrict__ nblocks_dev, int64_t max_blocks,
-                               int32_t* __restrict__ nz_begin, int32_t* __restrict__ nz_end,
+                               const int32_t* __restrict__ brp, const int32_t* __restrict__ bcol, int nseg,
+                               const int64_t* __restrict__ seg, const int32_t* __restrict__ nblocks_dev,
+                               int64_t max_blocks, int32_t* __restrict__ nz_begin, int32_t* __restrict__ nz_end,
                                int64_t* __restrict__ products, int64_t* __restrict__ slots,
-                               int32_t* __restrict__ hash_ok) {
+                               int32_t* __restrict__ hash_ok, int64_t* __restrict__ ncand) {
   __shared__ int64_t s_nz[SEG_STRIDE], s_base[SEG_STRIDE];
+  __shared__ int s_cand;
   for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
     s_nz[i] = seg[SEG_STRIDE + i];
     s_base[i] = seg[2 * SEG_STRIDE + i];
   }
+  if (threadIdx.x == 0) s_cand = 0;
   __syncthreads();
   const int64_t b = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
-  if (b >= max_blocks) return;
   const int nblocks = *nblocks_dev;
-  if (b >= nblocks) {
-    if (lane == 0) {
-      products[b] = 0; slots[b] = 0; nz_begin[b] = 0; nz_end[b] = 0;
-      if (hash_ok) hash_ok[b] = 0;
+  if (b < max_blocks && b >= nblocks && lane == 0) {
+    products[b] = 0; slots[b] = 0; nz_begin[b] = 0; nz_end[b] = 0;
+    if (hash_ok) hash_ok[b] = 0;
+  }
+  if (b < nblocks) {
+    int s = 0;
+    while (s + 1 < nseg && s_base[s + 1] <= b) ++s;
+    const int64_t nzb = s_nz[s] + (b - s_base[s]) * NPB;
+    const int64_t nze = min(nzb + (int64_t)NPB, s_nz[s + 1]);
+    int64_t sum = 0, waves = 0;
+    for (int64_t p = nzb + lane; p < nze; p += 32) {
+      const int k = acol[p];
+      const int len = brp[k + 1] - brp[k];
+      sum += len;
+      waves += (len + 31) >> 5;
     }
-    return;
-  }
-  int s = 0;
-  while (s + 1 < nseg && s_base[s + 1] <= b) ++s;
-  const int64_t nzb = s_nz[s] + (b - s_base[s]) * NPB;
-  const int64_t nze = min(nzb + (int64_t)NPB, s_nz[s + 1]);
-  int64_t sum = 0, waves = 0;
-  for (int64_t p = nzb + lane; p < nze; p += 32) {
-    const int k = acol[p];
-    const int len = brp[k + 1] - brp[k];
-    sum += len;
-    waves += (len + 31) >> 5;
-  }
 #pragma unroll
-  for (int d = 16; d > 0; d >>= 1) {
-    sum += __shfl_xor_sync(0xffffffffu, sum, d);
-    waves += __shfl_xor_sync(0xffffffffu, waves, d);
-  }
-  // hash accumulator candidate (reading R31), two deterministic tests on the block's own
-  // entries: (1) its waves (one entry x <= 32 entries of the entry's B row) keep at least
-  // half of the lanes busy -- short B rows stay in AC-ESC, whose draws pack them
-  // densely; (2) the rows are likely to compact: the B rows of adjacent entries share at
-  // least a quarter of their columns (8 sampled pairs, first <= 32 columns of each) --
-  // random-column rows barely compact, and AC-ESC's sort is cheaper than hashing and
-  // then sorting them
-  int hok = 0;
-  if (hash_ok && sum > 0 && 2 * sum >= 32 * waves) {
-    constexpr int NS = 8;                     // sampled adjacent pairs
-    const int64_t n = nze - nzb;
-    int ov = 0, mn = 0;
-    if (n >= 2) {
-      int v1[NS], v2[NS], l1[NS], l2[NS];
+    for (int d = 16; d > 0; d >>= 1) {
+      sum += __shfl_xor_sync(0xffffffffu, sum, d);
+      waves += __shfl_xor_sync(0xffffffffu, waves, d);
+    }
+    int hok = 0;
+    if (hash_ok && sum > 0 && 2 * sum >= 32 * waves) {
+      constexpr int NS = 8;                   // sampled adjacent pairs
+      const int64_t n = nze - nzb;
+      int ov = 0, mn = 0;
+      if (n >= 2) {
+        int v1[NS], v2[NS], l1[NS], l2[NS];
 #pragma unroll
-      for (int s = 0; s < NS; ++s) {
-        const int64_t p = nzb + ((int64_t)s * (n - 1)) / NS;
-        const int k1 = acol[p], k2 = acol[p + 1];
-        const int a0 = brp[k1], b0 = brp[k2];
-        l1[s] = min(brp[k1 + 1] - a0, 32);
-        l2[s] = min(brp[k2 + 1] - b0, 32);
-        v1[s] = lane < l1[s] ? bcol[a0 + lane] : INT_MAX;
-        v2[s] = lane < l2[s] ? bcol[b0 + lane] : INT_MAX;
-      }
-#pragma unroll
-      for (int s = 0; s < NS; ++s) {
-        // position of v1 among the sorted v2 (held across the lanes): count of v2 < v1
-        int pos = 0;
-#pragma unroll
-        for (int step = 16; step > 0; step >>= 1) {
-          const int x = __shfl_sync(0xffffffffu, v2[s], pos + step - 1);
-          if (x < v1[s]) pos += step;
+        for (int q = 0; q < NS; ++q) {
+          const int64_t p = nzb + ((int64_t)q * (n - 1)) / NS;
+          const int k1 = acol[p], k2 = acol[p + 1];
+          const int a0 = brp[k1], b0 = brp[k2];
+          l1[q] = min(brp[k1 + 1] - a0, 32);
+          l2[q] = min(brp[k2 + 1] - b0, 32);
+          v1[q] = lane < l1[q] ? bcol[a0 + lane] : INT_MAX;
+          v2[q] = lane < l2[q] ? bcol[b0 + lane] : INT_MAX;
         }
-        const int at = __shfl_sync(0xffffffffu, v2[s], pos & 31);
-        ov += lane < l1[s] && pos < 32 && at == v1[s];
-        mn += min(l1[s], l2[s]);
+#pragma unroll
+        for (int q = 0; q < NS; ++q) {
+          // position of v1 among the sorted v2 (held across the lanes): count of v2 < v1
+          int pos = 0;
+#pragma unroll
+          for (int step = 16; step > 0; step >>= 1) {
+            const int x = __shfl_sync(0xffffffffu, v2[q], pos + step - 1);
+            if (x < v1[q]) pos += step;
+          }
+          const int at = __shfl_sync(0xffffffffu, v2[q], pos & 31);
+          ov += lane < l1[q] && pos < 32 && at == v1[q];
+          mn += min(l1[q], l2[q]);
+        }
       }
+      ov = __reduce_add_sync(0xffffffffu, ov);
+      hok = mn > 0 && 4 * ov >= mn;
     }
-    ov = __reduce_add_sync(0xffffffffu, ov);
-    hok = mn > 0 && 4 * ov >= mn;
+    if (lane == 0) {
+      if (hash_ok) hash_ok[b] = hok;
+      if (hok) atomicAdd(&s_cand, 1);
+      products[b] = sum;
+      // the hash accumulator (R31) emits up to one chunk per warp
+      slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)HASH_WARPS) : 0;
+      nz_begin[b] = (int32_t)nzb;
+      nz_end[b] = (int32_t)nze;
+    }
   }
-  if (lane == 0) {
-    if (hash_ok) hash_ok[b] = hok;
-    products[b] = sum;
-    // the hash accumulator (R31) emits up to one chunk per warp
-    slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)HASH_WARPS) : 0;
-    nz_begin[b] = (int32_t)nzb;
-    nz_end[b] = (int32_t)nze;
-  }
+  __syncthreads();
+  if (threadIdx.x == 0 && ncand && s_cand)
+    atomicAdd(reinterpret_cast<unsigned long long*>(ncand), (unsigned long long)s_cand);
 }
 
 void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* nzb, int32_t* nze,
-                         int64_t* products, int64_t* slots, int32_t* hash_ok, cudaStream_t st) {
+                         int64_t* products, int64_t* slots, int32_t* hash_ok, int64_t* ncand, cudaStream_t st) {
   if (max_blocks == 0) return;
   const int T = 256, WPB = T / 32;
   k_block_bounds<<<(unsigned)((max_blocks + WPB - 1) / WPB), T, 0, st>>>(
-      A.row_ptr, A.col, B.row_ptr, B.col, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots, hash_ok);
+      A.row_ptr, A.col, B.row_ptr, B.col, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots, hash_ok,
+      ncand);
 }
 
 // Canonical-CSR check (reading R3): row_ptr monotone, columns strictly increasing and

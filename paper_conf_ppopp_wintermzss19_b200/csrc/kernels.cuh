@@ -23,7 +23,8 @@ void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* block_r
 void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* blk_nz_begin,
                          int32_t* blk_nz_end, int64_t* blk_products, int64_t* blk_slots,
-                         int32_t* blk_hash_ok /* nullable: hash-accumulator candidates (R31) */, cudaStream_t st);
+                         int32_t* blk_hash_ok /* nullable: hash-accumulator candidates (R31) */,
+                         int64_t* ncand /* nullable: their count (zeroed by the caller) */, cudaStream_t st);
 
 // ---- device-wide exclusive scan (scan.cu) --------------------------------------
 // out[i] = sum_{j<i} in[j] for i < n, total -> *total_dev.  tmp needs scan_tmp_elems(n).

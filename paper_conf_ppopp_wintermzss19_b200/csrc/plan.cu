@@ -254,9 +254,10 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   tl_launches += 1;
   launch_glb(Av, nseg, ptr<int64_t>(p->seg), ptr<int32_t>(p->brs), max_blocks, st);
   tl_launches += 1;
+  ACS_CUDA(cudaMemsetAsync(scal + 3, 0, sizeof(int64_t), st));   // hash candidates (R31)
   launch_block_bounds(Av, Bv, nseg, ptr<int64_t>(p->seg), nblocks_dev, max_blocks, ptr<int32_t>(p->nzb),
                       ptr<int32_t>(p->nze), ptr<int64_t>(p->bprod), ptr<int64_t>(p->bslot),
-                      p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE ? ptr<int32_t>(p->hdone) : nullptr, st);
+                      p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE ? ptr<int32_t>(p->hdone) : nullptr, scal + 3, st);
   tl_launches += 1;
   launch_scan_i64(ptr<int64_t>(p->bprod), ptr<int64_t>(p->pool_off), max_blocks, scal + 0, ptr<int64_t>(p->scan_tmp), st);
   launch_scan_i64(ptr<int64_t>(p->bslot), ptr<int64_t>(p->desc_off), max_blocks, scal + 1, ptr<int64_t>(p->scan_tmp), st);
@@ -267,8 +268,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   // segment boundaries (for info) ride along with the first read-back
   launch_read_back(p->seg.p, p->h_scal + H_SEG_INFO, (int)sizeof(int64_t) * (nseg + 1), st);
   tl_launches += 1;
-  if ((s = sync_read(p, scal, 3, st)) != ACSPGEMM_OK) return s;
-  const int64_t products = p->h_scal[0], slots = p->h_scal[1], nblocks = p->h_scal[2];
+  if ((s = sync_read(p, scal, 4, st)) != ACSPGEMM_OK) return s;
+  const int64_t products = p->h_scal[0], slots = p->h_scal[1], nblocks = p->h_scal[2], ncand = p->h_scal[3];
   p->info.products = products;
   p->info.nblocks = nblocks;
   p->info.nsegments = nseg;
@@ -320,8 +321,10 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     ACS_CUDA(cudaMemsetAsync(scal + 30, 0, 2 * sizeof(int64_t), st));
     ea.hash_done = ptr<int32_t>(p->hdone);
     ea.esc_list_small = ptr<int32_t>(p->esc_list_small);
-    launch_hash(ea, p->f64, st);
-    tl_launches += nblocks > 0 ? 1 : 0;
+    if (ncand > 0) {
+      launch_hash(ea, p->f64, st);
+      tl_launches += nblocks > 0 ? 1 : 0;
+    }
   }
   record(p, S_HASHEND, st);
   if (ea.hash_done) {
