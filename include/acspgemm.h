@@ -83,13 +83,17 @@ typedef struct {
   int validate_inputs;       /* 1: check that A and B are canonical CSR (one extra sync) */
   int collect_stage_times;   /* 1: record CUDA events between stages (acspgemm_stage_times) */
   int num_segments;          /* canonical segments S (default 8, max 64) */
-  int strategy;              /* ACSPGEMM_STRATEGY_ADAPTIVE (default): each block is tried by the
-                                hash accumulator first and falls back to AC-ESC (reading R31);
-                                ACSPGEMM_STRATEGY_ESC: every block through AC-ESC */
+  int strategy;              /* ACSPGEMM_STRATEGY_ADAPTIVE (default): each candidate block is tried
+                                by the column-dictionary accumulator (reading R33), then the hash
+                                accumulator (R31), and falls back to AC-ESC;
+                                ACSPGEMM_STRATEGY_ESC: every block through AC-ESC;
+                                ACSPGEMM_STRATEGY_HASH: as ADAPTIVE without the dictionary
+                                accumulator (same results bit for bit; for comparison) */
 } acspgemm_options;
 
 #define ACSPGEMM_STRATEGY_ADAPTIVE 0
 #define ACSPGEMM_STRATEGY_ESC 1
+#define ACSPGEMM_STRATEGY_HASH 2
 
 /* Counters of the last multiply of a plan (host values). */
 typedef struct {
@@ -107,7 +111,8 @@ typedef struct {
   int64_t kernel_launches;   /* kernels launched by the last symbolic + numeric */
   int32_t nsegments;
   int64_t segment_rows[65];
-  int64_t nhash_blocks;      /* blocks completed by the hash accumulator (strategy ADAPTIVE) */
+  int64_t nhash_blocks;      /* blocks completed by an accumulator (dictionary or hash; R33, R31) */
+  int64_t ndict_blocks;      /* of them, blocks completed by the column-dictionary accumulator (R33) */
 } acspgemm_info;
 
 /* Defaults: no pool limit, no validation, no stage times, 8 segments, adaptive strategy. */

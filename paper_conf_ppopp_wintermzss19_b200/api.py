@@ -81,15 +81,19 @@ def _stream_ptr(stream: Optional[torch.cuda.Stream]) -> ctypes.c_void_p:
     return ctypes.c_void_p(s.cuda_stream)
 
 
+_STRATEGIES = {"adaptive": 0, "esc": 1, "hash": 2}   # ACSPGEMM_STRATEGY_* (include/acspgemm.h)
+
+
 class Plan:
     """A reusable multiply plan (owns the chunk pool and helper memory)."""
 
     def __init__(self, pool_limit_bytes: int = 0, validate: bool = False, stage_times: bool = False,
                  num_segments: int = 8, strategy: str = "adaptive"):
-        """strategy: "adaptive" (hash accumulator per block, AC-ESC fallback; reading R31)
-        or "esc" (every block through AC-ESC)."""
-        if strategy not in ("adaptive", "esc"):
-            raise ValueError("strategy must be 'adaptive' or 'esc'")
+        """strategy: "adaptive" (column-dictionary accumulator, then hash accumulator per
+        candidate block, AC-ESC fallback; readings R33, R31), "hash" (as adaptive without
+        the dictionary accumulator: the same bits) or "esc" (every block through AC-ESC)."""
+        if strategy not in _STRATEGIES:
+            raise ValueError("strategy must be 'adaptive', 'esc' or 'hash'")
         lib = load()
         opt = Options()
         lib.acspgemm_options_default(ctypes.byref(opt))
@@ -97,7 +101,7 @@ class Plan:
         opt.validate_inputs = int(bool(validate))
         opt.collect_stage_times = int(bool(stage_times))
         opt.num_segments = int(num_segments)
-        opt.strategy = 0 if strategy == "adaptive" else 1
+        opt.strategy = _STRATEGIES[strategy]
         h = ctypes.c_void_p()
         check(lib.acspgemm_plan_create(ctypes.byref(h), ctypes.byref(opt)), "acspgemm_plan_create")
         self._h = h

@@ -14,7 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 BUILD = os.path.join(HERE, "build")
 SO = os.path.join(HERE, "libacspgemm.so")
-SOURCES = ["glb.cu", "scan.cu", "esc.cu", "esc_small.cu", "hash.cu", "merge.cu", "copy.cu", "plan.cu"]
+SOURCES = ["glb.cu", "scan.cu", "esc.cu", "esc_small.cu", "hash.cu", "dict.cu", "merge.cu", "copy.cu", "plan.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr", "-ftz=false", "-prec-div=true",

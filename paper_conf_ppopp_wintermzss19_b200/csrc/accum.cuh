@@ -1,0 +1,163 @@
+// Shared pieces of the per-block accumulators of the adaptive strategy (hash.cu,
+// reading R31; dict.cu, reading R33): exact IEEE product/sum and Fetch A.
+#pragma once
+#include <climits>
+#include "kernels.cuh"
+
+namespace acs {
+
+__device__ __forceinline__ float vmul(float x, float y) { return __fmul_rn(x, y); }
+__device__ __forceinline__ double vmul(double x, double y) { return __dmul_rn(x, y); }
+__device__ __forceinline__ float vadd(float x, float y) { return __fadd_rn(x, y); }
+__device__ __forceinline__ double vadd(double x, double y) { return __dadd_rn(x, y); }
+
+// Fetch A (§3.2.1) for one block of NPB nonzeros, as in AC-ESC, by THREADS
+// threads:
+//   * entries whose B row is empty add no products and are dropped; the others are
+//     compacted in storage order: ent[ci].x = B row start, ent[ci].y = its length,
+//     a_val[ci] = A value, wd[ci] = exclusive product prefix (the WDState of Alg. 2),
+//     wd[nent] = the block's products;
+//   * the block's rows are numbered by rank: row_first[lr] = first compacted entry of
+//     local row lr (row_first[nrows] = nent), row_of[lr] = the row of A (and C).
+// rp_cache needs NPB + 1 ints and may alias other storage after the call; scratch needs
+// THREADS/32 + 1 ints.  Ends with a __syncthreads().  Returns whether this thread saw a
+// B row longer than 32 entries.
+template <typename T, typename E>
+__device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cache, int* row_of, int* row_first,
+                                            E* ent, T* a_val, int* wd, int* scratch, int& nrows, int& nent,
+                                            int& total) {
+  const int tid = threadIdx.x;
+  const int32_t* __restrict__ arp = a.A.row_ptr;
+  const int32_t* __restrict__ acol = a.A.col;
+  const T* __restrict__ aval = reinterpret_cast<const T*>(a.A.val);
+  const int32_t* __restrict__ brp = a.B.row_ptr;
+  const int nzb = a.blk_nz_begin[b];
+  const int n_a = a.blk_nz_end[b] - nzb;
+  const int r0 = a.block_row_starts[b];
+  const int64_t rowsA = a.A.rows;
+  for (int t = tid; t <= NPB; t += THREADS) {
+    const int64_t r = (int64_t)r0 + t;
+    rp_cache[t] = r <= rowsA ? arp[r] : INT_MAX;
+  }
+  __syncthreads();
+  int len[NNZ_PER_THREAD], row[NNZ_PER_THREAD], bst[NNZ_PER_THREAD];
+  T av[NNZ_PER_THREAD];
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+    const int e = tid * NNZ_PER_THREAD + j;
+    len[j] = 0;
+    row[j] = INT_MAX;
+    bst[j] = 0;
+    av[j] = (T)0;
+    if (e < n_a) {
+      const int nz = nzb + e;
+      const int k = acol[nz];
+      av[j] = aval[nz];
+      bst[j] = brp[k];
+      len[j] = brp[k + 1] - bst[j];
+      int r;
+      if (nz < rp_cache[NPB]) {
+        int lo = 0, hi = NPB - 1;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (rp_cache[mid] <= nz) lo = mid; else hi = mid - 1;
+        }
+        r = r0 + lo;
+      } else {
+        int64_t lo = (int64_t)r0 + NPB, hi = rowsA - 1;
+        while (lo < hi) {
+          const int64_t mid = (lo + hi + 1) >> 1;
+          if (arp[mid] <= nz) lo = mid; else hi = mid - 1;
+        }
+        r = (int)lo;
+      }
+      row[j] = r;
+    }
+    row_of[e] = row[j];        // temporarily: row per entry
+  }
+  __syncthreads();
+  // one packed scan numbers the rows (low 16 bits) and the nonempty entries (high 16)
+  int f[NNZ_PER_THREAD], packed = 0, psum = 0;
+  bool longb = false;
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+    const int e = tid * NNZ_PER_THREAD + j;
+    f[j] = (e < n_a) && (e == 0 || row_of[e - 1] != row[j]);
+    packed += f[j] + ((len[j] > 0) << 16);
+    psum += len[j];
+    longb |= len[j] > 32;
+  }
+  int tot_packed;
+  int ex = block_exclusive_sum<int>(packed, scratch, &tot_packed);   // barriers: reads above done
+  int pex = block_exclusive_sum<int>(psum, scratch, &total);
+  nrows = tot_packed & 0xFFFF;
+  nent = tot_packed >> 16;
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+    const int lr = ex & 0xFFFF, ci = ex >> 16;
+    if (f[j]) {
+      row_first[lr] = ci;
+      row_of[lr] = row[j];
+    }
+    if (len[j] > 0) {
+      ent[ci].x = bst[j];
+      ent[ci].y = len[j];
+      a_val[ci] = av[j];
+      wd[ci] = pex;
+    }
+    ex += f[j] + ((len[j] > 0) << 16);
+    pex += len[j];
+  }
+  if (tid == 0) {
+    row_first[nrows] = nent;
+    wd[nent] = total;
+  }
+  __syncthreads();
+  return longb;
+}
+
+// Rows -> warps by product count: warp w of NW owns the rows whose first product lies in
+// [w·P/NW, (w+1)·P/NW).  Lane 0 of each warp writes wrow[w] (wrow[NW] = nrows); the
+// caller synchronises.
+template <int NW>
+__device__ __forceinline__ void split_rows(const int* wd, const int* row_first, int nrows, int total, int* wrow) {
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) {
+    const int L = (int)((int64_t)w * total / NW);
+    int lo = 0, hi = nrows;              // first r with start(r) >= L
+    while (lo < hi) {
+      const int mid = (lo + hi) >> 1;
+      if (wd[row_first[mid]] < L) lo = mid + 1; else hi = mid;
+    }
+    wrow[w] = w == 0 ? 0 : lo;
+    if (w == NW - 1) wrow[NW] = nrows;
+  }
+}
+
+// One chunk descriptor per warp that emitted rows (L424-L428), in warp order = row
+// order; wout[q] = {count, first_row, last_row, first_count, last_count}.  Thread 0.
+__device__ __forceinline__ void emit_warp_chunks(const EscArgs& a, int b, int nw, const int* wrow, const int (*wout)[5],
+                                                 const int* wd, const int* row_first) {
+  const int64_t pool_base = a.pool_off[b];
+  const int64_t desc_base = a.desc_off[b];
+  int seq = 0, used = 0;
+  for (int q = 0; q < nw; ++q) {
+    if (wout[q][0] == 0) continue;
+    ChunkDesc d;
+    d.data_off = pool_base + wd[row_first[wrow[q]]];
+    d.first_row = wout[q][1];
+    d.last_row = wout[q][2];
+    d.count = wout[q][0];
+    d.first_count = wout[q][3];
+    d.last_count = wout[q][4];
+    d.flags = 0;
+    a.descs[desc_base + seq] = d;
+    ++seq;
+    used += wout[q][0];
+  }
+  a.nchunks[b] = seq;
+  a.used[b] = used;
+  atomicAdd(reinterpret_cast<unsigned long long*>(a.hash_count), 1ull);
+}
+
+}  // namespace acs

@@ -257,7 +257,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_CUDA(cudaMemsetAsync(scal + 3, 0, sizeof(int64_t), st));   // hash candidates (R31)
   launch_block_bounds(Av, Bv, nseg, ptr<int64_t>(p->seg), nblocks_dev, max_blocks, ptr<int32_t>(p->nzb),
                       ptr<int32_t>(p->nze), ptr<int64_t>(p->bprod), ptr<int64_t>(p->bslot),
-                      p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE ? ptr<int32_t>(p->hdone) : nullptr, scal + 3, st);
+                      p->opt.strategy != ACSPGEMM_STRATEGY_ESC ? ptr<int32_t>(p->hdone) : nullptr, scal + 3, st);
   tl_launches += 1;
   launch_scan_i64(ptr<int64_t>(p->bprod), ptr<int64_t>(p->pool_off), max_blocks, scal + 0, ptr<int64_t>(p->scan_tmp), st);
   launch_scan_i64(ptr<int64_t>(p->bslot), ptr<int64_t>(p->desc_off), max_blocks, scal + 1, ptr<int64_t>(p->scan_tmp), st);
@@ -306,22 +306,27 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.row_count = ptr<int32_t>(p->row_count);
   ea.hash_done = nullptr;
   ea.hash_count = scal + 6;
+  ea.dict_count = scal + 7;
   ea.esc_list = ptr<int32_t>(p->esc_list);
   ea.esc_count = scal + 28;
   ea.esc_next = scal + 29;
-  ACS_CUDA(cudaMemsetAsync(scal + 6, 0, sizeof(int64_t), st));
+  ACS_CUDA(cudaMemsetAsync(scal + 6, 0, 2 * sizeof(int64_t), st));
   ACS_CUDA(cudaMemsetAsync(scal + 28, 0, 2 * sizeof(int64_t), st));
   ea.blk_products = ptr<int64_t>(p->bprod);
   ea.esc_list_small = nullptr;
   ea.esc_count_small = scal + 30;
   ea.esc_next_small = scal + 31;
-  if (p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE) {
+  if (p->opt.strategy != ACSPGEMM_STRATEGY_ESC) {
     // hash accumulator first (reading R31); blocks it does not finish go to AC-ESC,
     // small ones (<= 512 products) to the small-tile AC-ESC (reading R32)
     ACS_CUDA(cudaMemsetAsync(scal + 30, 0, 2 * sizeof(int64_t), st));
     ea.hash_done = ptr<int32_t>(p->hdone);
     ea.esc_list_small = ptr<int32_t>(p->esc_list_small);
     if (ncand > 0) {
+      if (p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE) {
+        launch_dict(ea, p->f64, st);     // column dictionary first (reading R33)
+        tl_launches += nblocks > 0 ? 1 : 0;
+      }
       launch_hash(ea, p->f64, st);
       tl_launches += nblocks > 0 ? 1 : 0;
     }
@@ -363,8 +368,9 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   launch_find_shared(ms, scal + 4, st);
   tl_launches += 1 + (slots > 0 ? 5 : 0);
   ACS_CUDA(cudaGetLastError());
-  if ((s = sync_read(p, scal + 3, 4, st)) != ACSPGEMM_OK) return s;
+  if ((s = sync_read(p, scal + 3, 5, st)) != ACSPGEMM_OK) return s;
   p->info.nhash_blocks = p->h_scal[3];
+  p->info.ndict_blocks = p->h_scal[4];
   p->total_chunks = p->h_scal[0];
   p->nshared = p->h_scal[1];
   p->max_chunks = slots;
@@ -678,7 +684,8 @@ acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options
     delete p;
     return set_err(ACSPGEMM_ERR_INVALID_ARG, "num_segments > 64");
   }
-  if (p->opt.strategy != ACSPGEMM_STRATEGY_ADAPTIVE && p->opt.strategy != ACSPGEMM_STRATEGY_ESC) {
+  if (p->opt.strategy != ACSPGEMM_STRATEGY_ADAPTIVE && p->opt.strategy != ACSPGEMM_STRATEGY_ESC &&
+      p->opt.strategy != ACSPGEMM_STRATEGY_HASH) {
     delete p;
     return set_err(ACSPGEMM_ERR_INVALID_ARG, "unknown strategy");
   }
