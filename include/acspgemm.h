@@ -84,16 +84,18 @@ typedef struct {
   int collect_stage_times;   /* 1: record CUDA events between stages (acspgemm_stage_times) */
   int num_segments;          /* canonical segments S (default 8, max 64) */
   int strategy;              /* ACSPGEMM_STRATEGY_ADAPTIVE (default): each candidate block is tried
-                                by the column-dictionary accumulator (reading R33), then the hash
-                                accumulator (R31), and falls back to AC-ESC;
+                                by the column-dictionary accumulator (reading R33; fp32 only),
+                                then the hash accumulator (R31), and falls back to AC-ESC;
                                 ACSPGEMM_STRATEGY_ESC: every block through AC-ESC;
-                                ACSPGEMM_STRATEGY_HASH: as ADAPTIVE without the dictionary
-                                accumulator (same results bit for bit; for comparison) */
+                                ACSPGEMM_STRATEGY_HASH: hash accumulator, then AC-ESC;
+                                ACSPGEMM_STRATEGY_DICT: dictionary (any dtype), hash, AC-ESC.
+                                ADAPTIVE, HASH and DICT give the same results bit for bit. */
 } acspgemm_options;
 
 #define ACSPGEMM_STRATEGY_ADAPTIVE 0
 #define ACSPGEMM_STRATEGY_ESC 1
 #define ACSPGEMM_STRATEGY_HASH 2
+#define ACSPGEMM_STRATEGY_DICT 3
 
 /* Counters of the last multiply of a plan (host values). */
 typedef struct {
@@ -183,8 +185,9 @@ acspgemm_status acspgemm_free_csr(acspgemm_csr_out* C, void* stream);
 
 /* Per-stage device times (ms) of the last symbolic + numeric when collect_stage_times
  * was set, in the order of Fig. 7 (L740): GLB, ESC, MCC, MM, PM, SM, SCAN, CC, then HASH:
- * the part of ESC spent in the hash accumulator (strategy ADAPTIVE, reading R31).
- * Writes min(n, 9) values.  Synchronises the plan's events. */
+ * the part of ESC spent in the accumulators (column dictionary + hash table, readings
+ * R33, R31), then DICT: the part spent in the column-dictionary accumulator.
+ * Writes min(n, 10) values.  Synchronises the plan's events. */
 acspgemm_status acspgemm_stage_times(acspgemm_plan plan, float* ms_out, int n);
 
 /* Counters of the last multiply. */

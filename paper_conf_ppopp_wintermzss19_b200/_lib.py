@@ -9,7 +9,8 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(HERE, "libacspgemm.so")
+# ACSPGEMM_LIB: an in-tree build variant (e.g. libacspgemm_w4.so from build.py with ACS_BUILD_TAG)
+SO_PATH = os.environ.get("ACSPGEMM_LIB") or os.path.join(HERE, "libacspgemm.so")
 
 I32, I64, U32 = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32
 VP = ctypes.c_void_p

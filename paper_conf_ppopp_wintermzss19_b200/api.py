@@ -16,7 +16,8 @@ from . import _lib
 from ._lib import CsrIn, CsrOut, Info, Options, check, load
 
 F32, F64 = 0, 1
-STAGES = ("GLB", "ESC", "MCC", "MM", "PM", "SM", "SCAN", "CC", "HASH")   # HASH: k_hash part of ESC
+# HASH: the accumulator part of ESC (k_dict + k_hash); DICT: its k_dict part
+STAGES = ("GLB", "ESC", "MCC", "MM", "PM", "SM", "SCAN", "CC", "HASH", "DICT")
 
 
 @dataclass
@@ -81,7 +82,7 @@ def _stream_ptr(stream: Optional[torch.cuda.Stream]) -> ctypes.c_void_p:
     return ctypes.c_void_p(s.cuda_stream)
 
 
-_STRATEGIES = {"adaptive": 0, "esc": 1, "hash": 2}   # ACSPGEMM_STRATEGY_* (include/acspgemm.h)
+_STRATEGIES = {"adaptive": 0, "esc": 1, "hash": 2, "dict": 3}   # ACSPGEMM_STRATEGY_* (include/acspgemm.h)
 
 
 class Plan:
@@ -89,11 +90,12 @@ class Plan:
 
     def __init__(self, pool_limit_bytes: int = 0, validate: bool = False, stage_times: bool = False,
                  num_segments: int = 8, strategy: str = "adaptive"):
-        """strategy: "adaptive" (column-dictionary accumulator, then hash accumulator per
-        candidate block, AC-ESC fallback; readings R33, R31), "hash" (as adaptive without
-        the dictionary accumulator: the same bits) or "esc" (every block through AC-ESC)."""
+        """strategy: "adaptive" (column-dictionary accumulator for fp32, then the hash
+        accumulator per candidate block, AC-ESC fallback; readings R33, R31), "hash" (no
+        dictionary), "dict" (dictionary for every dtype) -- these three give the same bits --
+        or "esc" (every block through AC-ESC)."""
         if strategy not in _STRATEGIES:
-            raise ValueError("strategy must be 'adaptive', 'esc' or 'hash'")
+            raise ValueError("strategy must be one of " + ", ".join(_STRATEGIES))
         lib = load()
         opt = Options()
         lib.acspgemm_options_default(ctypes.byref(opt))

@@ -12,8 +12,10 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-BUILD = os.path.join(HERE, "build")
-SO = os.path.join(HERE, "libacspgemm.so")
+# ACS_BUILD_TAG builds a variant (with ACS_EXTRA_NVCC_FLAGS) into build_<tag>/libacspgemm_<tag>.so
+_TAG = os.environ.get("ACS_BUILD_TAG", "")
+BUILD = os.path.join(HERE, "build" + (f"_{_TAG}" if _TAG else ""))
+SO = os.path.join(HERE, "libacspgemm" + (f"_{_TAG}" if _TAG else "") + ".so")
 SOURCES = ["glb.cu", "scan.cu", "esc.cu", "esc_small.cu", "hash.cu", "dict.cu", "merge.cu", "copy.cu", "plan.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",

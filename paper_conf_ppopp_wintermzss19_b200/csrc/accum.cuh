@@ -11,8 +11,36 @@ __device__ __forceinline__ double vmul(double x, double y) { return __dmul_rn(x,
 __device__ __forceinline__ float vadd(float x, float y) { return __fadd_rn(x, y); }
 __device__ __forceinline__ double vadd(double x, double y) { return __dadd_rn(x, y); }
 
-// Fetch A (§3.2.1) for one block of NPB nonzeros, as in AC-ESC, by THREADS
-// threads:
+// Block-wide exclusive prefix sum for a CTA of NT threads (the fixed shuffle tree of
+// common.cuh's block_exclusive_sum).  `scratch` needs NT/32 + 1 elements.  Two
+// __syncthreads().
+template <int NT, typename V>
+__device__ __forceinline__ V block_exclusive_sum_nt(V x, V* scratch, V* total) {
+  constexpr int NW = NT / 32;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  V inc = x;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    V y = __shfl_up_sync(0xffffffffu, inc, d);
+    if (lane >= d) inc += y;
+  }
+  if (lane == 31) scratch[w] = inc;
+  __syncthreads();
+  V t = lane < NW ? scratch[lane] : (V)0;
+  V ti = t;
+#pragma unroll
+  for (int d = 1; d < NW; d <<= 1) {
+    V y = __shfl_up_sync(0xffffffffu, ti, d);
+    if (lane >= d) ti += y;
+  }
+  const V wpre = __shfl_sync(0xffffffffu, ti - t, w);
+  *total = __shfl_sync(0xffffffffu, ti, NW - 1);
+  __syncthreads();
+  return wpre + inc - x;
+}
+
+// Fetch A (§3.2.1) for one block of NPB nonzeros, as in AC-ESC, by NT
+// threads (default THREADS):
 //   * entries whose B row is empty add no products and are dropped; the others are
 //     compacted in storage order: ent[ci].x = B row start, ent[ci].y = its length,
 //     a_val[ci] = A value, wd[ci] = exclusive product prefix (the WDState of Alg. 2),
@@ -20,9 +48,9 @@ __device__ __forceinline__ double vadd(double x, double y) { return __dadd_rn(x,
 //   * the block's rows are numbered by rank: row_first[lr] = first compacted entry of
 //     local row lr (row_first[nrows] = nent), row_of[lr] = the row of A (and C).
 // rp_cache needs NPB + 1 ints and may alias other storage after the call; scratch needs
-// THREADS/32 + 1 ints.  Ends with a __syncthreads().  Returns whether this thread saw a
-// B row longer than 32 entries.
-template <typename T, typename E>
+// NT/32 + 1 ints.  Ends with a __syncthreads().  Returns whether this thread saw a B row
+// longer than 32 entries.
+template <typename T, typename E, int NT = THREADS>
 __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cache, int* row_of, int* row_first,
                                             E* ent, T* a_val, int* wd, int* scratch, int& nrows, int& nent,
                                             int& total) {
@@ -35,16 +63,18 @@ __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cac
   const int n_a = a.blk_nz_end[b] - nzb;
   const int r0 = a.block_row_starts[b];
   const int64_t rowsA = a.A.rows;
-  for (int t = tid; t <= NPB; t += THREADS) {
+  constexpr int NPT = NPB / NT;          // A entries per thread (blocked)
+  static_assert(NPB % NT == 0, "NPB must be a multiple of NT");
+  for (int t = tid; t <= NPB; t += NT) {
     const int64_t r = (int64_t)r0 + t;
     rp_cache[t] = r <= rowsA ? arp[r] : INT_MAX;
   }
   __syncthreads();
-  int len[NNZ_PER_THREAD], row[NNZ_PER_THREAD], bst[NNZ_PER_THREAD];
-  T av[NNZ_PER_THREAD];
+  int len[NPT], row[NPT], bst[NPT];
+  T av[NPT];
 #pragma unroll
-  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
-    const int e = tid * NNZ_PER_THREAD + j;
+  for (int j = 0; j < NPT; ++j) {
+    const int e = tid * NPT + j;
     len[j] = 0;
     row[j] = INT_MAX;
     bst[j] = 0;
@@ -77,23 +107,23 @@ __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cac
   }
   __syncthreads();
   // one packed scan numbers the rows (low 16 bits) and the nonempty entries (high 16)
-  int f[NNZ_PER_THREAD], packed = 0, psum = 0;
+  int f[NPT], packed = 0, psum = 0;
   bool longb = false;
 #pragma unroll
-  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
-    const int e = tid * NNZ_PER_THREAD + j;
+  for (int j = 0; j < NPT; ++j) {
+    const int e = tid * NPT + j;
     f[j] = (e < n_a) && (e == 0 || row_of[e - 1] != row[j]);
     packed += f[j] + ((len[j] > 0) << 16);
     psum += len[j];
     longb |= len[j] > 32;
   }
   int tot_packed;
-  int ex = block_exclusive_sum<int>(packed, scratch, &tot_packed);   // barriers: reads above done
-  int pex = block_exclusive_sum<int>(psum, scratch, &total);
+  int ex = block_exclusive_sum_nt<NT, int>(packed, scratch, &tot_packed);   // barriers: reads above done
+  int pex = block_exclusive_sum_nt<NT, int>(psum, scratch, &total);
   nrows = tot_packed & 0xFFFF;
   nent = tot_packed >> 16;
 #pragma unroll
-  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+  for (int j = 0; j < NPT; ++j) {
     const int lr = ex & 0xFFFF, ci = ex >> 16;
     if (f[j]) {
       row_first[lr] = ci;

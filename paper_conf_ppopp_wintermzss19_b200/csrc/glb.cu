@@ -183,8 +183,8 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
       if (hash_ok) hash_ok[b] = hok;
       if (hok) atomicAdd(&s_cand, 1);
       products[b] = sum;
-      // the hash accumulator (R31) emits up to one chunk per warp
-      slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)HASH_WARPS) : 0;
+      // the accumulators (R31, R33) emit up to one chunk per warp
+      slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)ACC_MAX_WARPS) : 0;
       nz_begin[b] = (int32_t)nzb;
       nz_end[b] = (int32_t)nze;
     }

@@ -60,8 +60,9 @@ struct DevBuf {
 constexpr int H_SEG_ROWS = 32;
 constexpr int H_SEG_INFO = H_SEG_ROWS + MAX_SEGMENTS + 1;
 constexpr int H_SCAL_WORDS = H_SEG_INFO + MAX_SEGMENTS + 1;
-// S_HASHEND: end of the hash-accumulator part of the ESC stage (stage 8 "HASH")
-enum Stage { S_GLB = 0, S_ESC, S_MCC, S_MM, S_PM, S_SM, S_SCAN, S_CC, S_END, S_HASHEND, NSTAGE_EV };
+// S_HASHEND: end of the accumulator part of the ESC stage (stage 8 "HASH": k_dict + k_hash);
+// S_DICTEND: end of its column-dictionary part (stage 9 "DICT": k_dict)
+enum Stage { S_GLB = 0, S_ESC, S_MCC, S_MM, S_PM, S_SM, S_SCAN, S_CC, S_END, S_HASHEND, S_DICTEND, NSTAGE_EV };
 
 }  // namespace
 
@@ -322,14 +323,20 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     ACS_CUDA(cudaMemsetAsync(scal + 30, 0, 2 * sizeof(int64_t), st));
     ea.hash_done = ptr<int32_t>(p->hdone);
     ea.esc_list_small = ptr<int32_t>(p->esc_list_small);
-    if (ncand > 0) {
-      if (p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE) {
-        launch_dict(ea, p->f64, st);     // column dictionary first (reading R33)
-        tl_launches += nblocks > 0 ? 1 : 0;
-      }
-      launch_hash(ea, p->f64, st);
-      tl_launches += nblocks > 0 ? 1 : 0;
-    }
+  }
+  // column dictionary first (reading R33): by default for fp32 only -- with fp64 values its
+  // per-warp accumulators allow 2 CTAs (16 warps) per SM and it measured slower than the
+  // hash table (cfg2: 10.5 vs 10.1 ms; fp32: 7.8 vs 9.5 ms); both give the same bits
+  const bool use_dict = p->opt.strategy == ACSPGEMM_STRATEGY_DICT ||
+                        (p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE && !p->f64);
+  if (ea.hash_done && ncand > 0 && use_dict) {
+    launch_dict(ea, p->f64, st);
+    tl_launches += nblocks > 0 ? 1 : 0;
+  }
+  record(p, S_DICTEND, st);
+  if (ea.hash_done && ncand > 0) {
+    launch_hash(ea, p->f64, st);         // blocks k_dict left (reading R31)
+    tl_launches += nblocks > 0 ? 1 : 0;
   }
   record(p, S_HASHEND, st);
   if (ea.hash_done) {
@@ -684,8 +691,7 @@ acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options
     delete p;
     return set_err(ACSPGEMM_ERR_INVALID_ARG, "num_segments > 64");
   }
-  if (p->opt.strategy != ACSPGEMM_STRATEGY_ADAPTIVE && p->opt.strategy != ACSPGEMM_STRATEGY_ESC &&
-      p->opt.strategy != ACSPGEMM_STRATEGY_HASH) {
+  if (p->opt.strategy < ACSPGEMM_STRATEGY_ADAPTIVE || p->opt.strategy > ACSPGEMM_STRATEGY_DICT) {
     delete p;
     return set_err(ACSPGEMM_ERR_INVALID_ARG, "unknown strategy");
   }
@@ -940,14 +946,14 @@ acspgemm_status acspgemm_stage_times(acspgemm_plan p, float* ms_out, int n) {
   if (!p || !ms_out) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
   if (!p->opt.collect_stage_times || !p->ev_ok) return set_err(ACSPGEMM_ERR_NOT_READY, "stage times not collected");
   if (p->empty) {
-    for (int i = 0; i < n && i < 9; ++i) ms_out[i] = 0.f;
+    for (int i = 0; i < n && i < 10; ++i) ms_out[i] = 0.f;
     return ACSPGEMM_OK;
   }
   ACS_CUDA(cudaEventSynchronize(p->ev[S_END]));
-  for (int i = 0; i < n && i < 9; ++i) {
+  for (int i = 0; i < n && i < 10; ++i) {
     float ms = 0.f;
-    // stage 8 (HASH) is the hash-accumulator part of stage 1 (ESC)
-    const int a = i < 8 ? i : (int)S_ESC, b = i < 8 ? i + 1 : (int)S_HASHEND;
+    // stages 8 (HASH: k_dict + k_hash) and 9 (DICT: k_dict) are parts of stage 1 (ESC)
+    const int a = i < 8 ? i : (int)S_ESC, b = i < 8 ? i + 1 : (i == 8 ? (int)S_HASHEND : (int)S_DICTEND);
     if (cudaEventElapsedTime(&ms, p->ev[a], p->ev[b]) != cudaSuccess) { cudaGetLastError(); ms = -1.f; }
     ms_out[i] = ms;
   }
