@@ -44,8 +44,12 @@ constexpr int GIANT_SLICE = 4096;            // columns per dense-slice CTA
 constexpr int DENSE_SPAN_RATIO = 16;         // dense slices when span <= 16 x pre-merge elements
 constexpr int PAIR_MAX = 512;
 // hash accumulator (hash.cu, reading R31)
-constexpr int HASH_WARPS = 4;                // warps per CTA; each emits one chunk per block
+#ifndef ACS_HASH_WARPS
+#define ACS_HASH_WARPS 4
+#endif
+constexpr int HASH_WARPS = ACS_HASH_WARPS;   // warps per CTA; each emits one chunk per block
 constexpr int ACC_MAX_WARPS = 8;             // most warps (= chunks) an accumulator uses per block (k_dict)
+static_assert(HASH_WARPS <= ACC_MAX_WARPS, "chunk slots per block (k_block_bounds)");
 constexpr int HASH_THREADS = 32 * HASH_WARPS;
 constexpr int HASH_T = 512;                  // table slots per warp
 constexpr int HASH_UMAX = 256;               // max distinct columns of a row (load <= 1/2)
