@@ -37,6 +37,17 @@ struct EscState {
   int64_t wofs;
 };
 
+// Staging slot of compacted element p.  Each thread emits ITEMS consecutive elements, so
+// the lanes of one store are ~ITEMS slots apart; a rotation inside every 32 (4-byte
+// columns) / 16 (8-byte values) slots by the row number spreads them over the banks,
+// and consecutive p (the coalesced read-out) stay conflict-free.  A permutation inside
+// each aligned group, so slots stay below CAP.
+__device__ __forceinline__ int stage_slot32(int p) { return (p & ~31) | ((p + (p >> 5)) & 31); }
+template <typename T>
+__device__ __forceinline__ int stage_slot(int p) {
+  return sizeof(T) == 8 ? ((p & ~15) | ((p + (p >> 4)) & 15)) : stage_slot32(p);
+}
+
 // Sort + compaction (Alg. 3) + emission of one local ESC iteration whose sort words are
 // already in s.words: completed rows become a chunk, the last row is kept.  Only the
 // key bits [IDXBITS, IDXBITS + sortbits) are sorted (0: words already sorted).
@@ -72,12 +83,12 @@ __device__ __forceinline__ void esc_tail(EscSmem<T>& S, const EscArgs& a, EscSta
   // chunk and merged later)
   const bool keep = size_after > 0 && rc_last <= KEEP;
   const int nchunk = total - (keep ? rc_last : 0);
-  // compacted element p goes to staging slot p: [0, nchunk) is the chunk, the kept
-  // row stays at [nchunk, total) for the next iteration
+  // compacted element p goes to staging slot stage_slot(p): [0, nchunk) is the chunk,
+  // the kept row stays at [nchunk, total) for the next iteration
   compaction_emit<Word, T>(k, ev, n, colbits, ctx, [&](int, Word key, T val, uint32_t state, bool row_end) {
     const int p = st_count(state) - 1;
-    stage_col[p] = colof(key, 0);
-    stage_val[p] = val;
+    stage_col[stage_slot32(p)] = colof(key, 0);
+    stage_val[stage_slot<T>(p)] = val;
     if (row_end && p < nchunk) {
       const int rc = st_row_count(state);
       const int rel = (int)(key >> colbits);
@@ -92,8 +103,8 @@ __device__ __forceinline__ void esc_tail(EscSmem<T>& S, const EscArgs& a, EscSta
     const int64_t dst = pool_base + st.wofs;
     T* pv = reinterpret_cast<T*>(a.pool_val);
     for (int p = tid; p < nchunk; p += THREADS) {
-      a.pool_col[dst + p] = stage_col[p];
-      pv[dst + p] = stage_val[p];
+      a.pool_col[dst + p] = stage_col[stage_slot32(p)];
+      pv[dst + p] = stage_val[stage_slot<T>(p)];
     }
     if (tid == 0) {
       ChunkDesc d;
@@ -113,8 +124,8 @@ __device__ __forceinline__ void esc_tail(EscSmem<T>& S, const EscArgs& a, EscSta
   st.kofs = nchunk;
   if (keep) {
     st.kept_lrow = rmin + lastrel;
-    st.kept_cmin = stage_col[nchunk];
-    st.kept_cmax = stage_col[total - 1];
+    st.kept_cmin = stage_col[stage_slot32(nchunk)];
+    st.kept_cmax = stage_col[stage_slot32(total - 1)];
   }
   __syncthreads();
 }
@@ -311,8 +322,8 @@ __device__ __forceinline__ void esc_block(EscSmem<T>& S, const EscArgs& a, const
     for (int j = 0; j < KEEP_PER_THREAD; ++j) {
       const int p = j * THREADS + tid;
       if (p < st.kept) {
-        kc[j] = reinterpret_cast<int*>(S.s.words)[st.kofs + p];
-        kv[j] = S.s.vals[st.kofs + p];
+        kc[j] = reinterpret_cast<int*>(S.s.words)[stage_slot32(st.kofs + p)];
+        kv[j] = S.s.vals[stage_slot<T>(st.kofs + p)];
       } else {
         kc[j] = 0;
         kv[j] = (T)0;
