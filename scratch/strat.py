@@ -9,7 +9,7 @@ dt = np.float64 if (len(sys.argv) < 2 or sys.argv[1] == "f64") else np.float32
 n = int(sys.argv[2]) if len(sys.argv) > 2 else 128
 A = poisson3d_27pt(n)
 dA = acs.DeviceCSR.from_host(A, "cuda", dt)
-for strat in ("adaptive", "hash"):
+for strat in (sys.argv[3].split(",") if len(sys.argv) > 3 else ("adaptive", "hash")):
     plan = acs.Plan(stage_times=True, strategy=strat)
     for _ in range(3): C = plan.multiply(dA, dA); del C
     torch.cuda.synchronize()
