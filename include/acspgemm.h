@@ -52,7 +52,7 @@ typedef enum {
   ACSPGEMM_OK = 0,
   ACSPGEMM_ERR_INVALID_ARG = 1,     /* null pointer with nnz > 0, negative size, non-canonical input */
   ACSPGEMM_ERR_DIM_MISMATCH = 2,    /* A.cols != B.rows */
-  ACSPGEMM_ERR_INDEX_OVERFLOW = 3,  /* nnz(C) >= 2^31 (int32 C.row_ptr) */
+  ACSPGEMM_ERR_INDEX_OVERFLOW = 3,  /* nnz(C) >= 2^31 with int32 C.row_ptr (acspgemm_numeric64 has none) */
   ACSPGEMM_ERR_OUT_OF_MEMORY = 4,   /* device allocation failed or pool_limit_bytes exceeded */
   ACSPGEMM_ERR_CUDA = 5,            /* a CUDA runtime error; see acspgemm_last_error() */
   ACSPGEMM_ERR_NOT_READY = 6,       /* acspgemm_numeric without a successful acspgemm_symbolic */
@@ -74,6 +74,14 @@ typedef struct {
   int32_t* col_idx;
   void* val;
 } acspgemm_csr_out;
+
+/* Output CSR with 64-bit row pointers (for nnz(C) >= 2^31; column indices stay int32). */
+typedef struct {
+  int64_t rows, cols, nnz;
+  int64_t* row_ptr;
+  int32_t* col_idx;
+  void* val;
+} acspgemm_csr_out64;
 
 typedef struct acspgemm_plan_s* acspgemm_plan;
 
@@ -147,8 +155,13 @@ acspgemm_status acspgemm_symbolic(acspgemm_plan plan, const acspgemm_csr_in* A, 
 
 /* Numeric pass: copy row_ptr and the chunk data into caller-allocated C
  * (row_ptr[rows+1], col_idx[nnz_c], val[nnz_c] of the dtype given to symbolic).
- * C->rows/cols/nnz are filled in.  Asynchronous on `stream`. */
+ * C->rows/cols/nnz are filled in.  Asynchronous on `stream`.  Returns
+ * ACSPGEMM_ERR_INDEX_OVERFLOW when nnz(C) >= 2^31 (int32 row_ptr): use acspgemm_numeric64. */
 acspgemm_status acspgemm_numeric(acspgemm_plan plan, acspgemm_csr_out* C, void* stream);
+
+/* Numeric pass into a C with int64 row_ptr[rows+1] (any nnz(C); outputs
+ * beyond 2^31 entries, e.g. skewed graph products).  Otherwise as acspgemm_numeric. */
+acspgemm_status acspgemm_numeric64(acspgemm_plan plan, acspgemm_csr_out64* C, void* stream);
 
 /* One-shot C = A·B.  The library allocates C->row_ptr/col_idx/val with cudaMallocAsync
  * on `stream`; release them with acspgemm_free_csr.  Uses a temporary plan. */

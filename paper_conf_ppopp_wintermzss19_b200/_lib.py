@@ -28,6 +28,10 @@ class CsrOut(ctypes.Structure):
                 ("row_ptr", VP), ("col_idx", VP), ("val", VP)]
 
 
+# acspgemm_csr_out64: the same layout (int64 row_ptr behind the pointer)
+CsrOut64 = CsrOut
+
+
 class Options(ctypes.Structure):
     _fields_ = [("pool_limit_bytes", ctypes.c_size_t), ("validate_inputs", ctypes.c_int),
                 ("collect_stage_times", ctypes.c_int), ("num_segments", ctypes.c_int),
@@ -52,6 +56,7 @@ SIGNATURES = {
     "acspgemm_canonical_segments": (ctypes.c_int, [ctypes.POINTER(CsrIn), ctypes.c_int, PI64, VP]),
     "acspgemm_symbolic": (ctypes.c_int, [VP, ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.c_int, VP, PI64]),
     "acspgemm_numeric": (ctypes.c_int, [VP, ctypes.POINTER(CsrOut), VP]),
+    "acspgemm_numeric64": (ctypes.c_int, [VP, ctypes.POINTER(CsrOut64), VP]),
     "acspgemm_multiply": (ctypes.c_int, [ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.POINTER(CsrOut), VP,
                                          ctypes.c_int]),
     "acspgemm_multiply_host": (ctypes.c_int, [VP, ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.c_int, VP,

@@ -13,7 +13,7 @@ import numpy as np
 import torch
 
 from . import _lib
-from ._lib import CsrIn, CsrOut, Info, Options, check, load
+from ._lib import AcspgemmError, CsrIn, CsrOut, Info, Options, check, load
 
 F32, F64 = 0, 1
 # HASH: the accumulator part of ESC (k_dict + k_hash); DICT: its k_dict part
@@ -22,7 +22,8 @@ STAGES = ("GLB", "ESC", "MCC", "MM", "PM", "SM", "SCAN", "CC", "HASH", "DICT")
 
 @dataclass
 class DeviceCSR:
-    """CSR matrix in CUDA memory: row_ptr/col int32, val float32 or float64."""
+    """CSR matrix in CUDA memory: row_ptr int32 (int64 for outputs of Plan.multiply(index64=True)),
+    col int32, val float32 or float64."""
     rows: int
     cols: int
     row_ptr: torch.Tensor
@@ -144,15 +145,24 @@ class Plan:
         return int(nnz.value)
 
     def numeric(self, row_ptr: torch.Tensor, col: torch.Tensor, val: torch.Tensor, stream=None) -> None:
+        """Numeric pass into caller-allocated C; an int64 row_ptr selects acspgemm_numeric64."""
         c = CsrOut(0, 0, 0, row_ptr.data_ptr(), col.data_ptr(), val.data_ptr())
-        check(self._lib.acspgemm_numeric(self._h, ctypes.byref(c), _stream_ptr(stream)), "acspgemm_numeric")
+        if row_ptr.dtype == torch.int64:
+            check(self._lib.acspgemm_numeric64(self._h, ctypes.byref(c), _stream_ptr(stream)), "acspgemm_numeric64")
+        elif row_ptr.dtype == torch.int32:
+            check(self._lib.acspgemm_numeric(self._h, ctypes.byref(c), _stream_ptr(stream)), "acspgemm_numeric")
+        else:
+            raise TypeError("row_ptr must be int32 or int64")
 
-    def multiply(self, A: DeviceCSR, B: DeviceCSR, stream=None, A_view=None) -> DeviceCSR:
-        """symbolic -> allocate C with torch on the device -> numeric."""
+    def multiply(self, A: DeviceCSR, B: DeviceCSR, stream=None, A_view=None, index64: bool = False) -> DeviceCSR:
+        """symbolic -> allocate C with torch on the device -> numeric.  index64: C.row_ptr
+        in int64 (required when nnz(C) >= 2^31; columns stay int32)."""
         nnz = self.symbolic(A, B, stream, A_view)
+        if not index64 and nnz >= 2 ** 31:
+            raise AcspgemmError(3, "Plan.multiply: nnz(C) >= 2^31 needs index64=True")   # INDEX_OVERFLOW
         dev = A.val.device
         rows = self._rows
-        rp = torch.empty(rows + 1, dtype=torch.int32, device=dev)
+        rp = torch.empty(rows + 1, dtype=torch.int64 if index64 else torch.int32, device=dev)
         col = torch.empty(max(nnz, 1), dtype=torch.int32, device=dev)
         val = torch.empty(max(nnz, 1), dtype=A.dtype, device=dev)
         self.numeric(rp, col, val, stream)

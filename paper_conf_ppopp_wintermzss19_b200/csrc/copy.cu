@@ -97,6 +97,31 @@ void launch_copy_offset(int32_t* dst, const int32_t* src, int64_t n, int32_t off
   k_copy_offset<<<grid, 256, 0, st>>>(dst, src, n, off);
 }
 
+// src == nullptr: dst[i] = off (the row pointers of an empty product)
+template <typename I>
+__global__ void k_rowptr_out(I* __restrict__ dst, const int64_t* __restrict__ src, int64_t n, I off) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = (src ? (I)src[i] : (I)0) + off;
+}
+
+void launch_rowptr_out(int32_t* dst, const int64_t* src, int64_t n, int32_t off, cudaStream_t st) {
+  if (n <= 0) return;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 148 * 8);
+  k_rowptr_out<int32_t><<<grid, 256, 0, st>>>(dst, src, n, off);
+}
+
+void launch_rowptr_out(int64_t* dst, const int64_t* src, int64_t n, int64_t off, cudaStream_t st) {
+  if (n <= 0) return;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 148 * 8);
+  k_rowptr_out<int64_t><<<grid, 256, 0, st>>>(dst, src, n, off);
+}
+
+__global__ void k_put_last(int64_t* row_ptr, int64_t n, const int64_t* total) { row_ptr[n] = *total; }
+
+void launch_put_last(int64_t* row_ptr, int64_t n, const int64_t* total, cudaStream_t st) {
+  k_put_last<<<1, 1, 0, st>>>(row_ptr, n, total);
+}
+
 __global__ void k_add_offset(int32_t* __restrict__ p, int64_t n, int32_t off) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     p[i] += off;

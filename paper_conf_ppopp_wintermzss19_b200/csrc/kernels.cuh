@@ -156,11 +156,17 @@ struct CopyArgs {
   const void* pool_val;
   const int32_t* merge_col;
   const void* merge_val;
-  const int32_t* row_ptr;
+  const int64_t* row_ptr;        // C's row pointers (plan memory, int64)
   int32_t* c_col;
   void* c_val;
 };
 void launch_copy(const CopyArgs& a, bool f64, cudaStream_t st);
+// C.row_ptr from the plan's int64 row pointers: dst[i] = src[i] + off (int32 or int64 dst;
+// src nullptr: dst[i] = off)
+void launch_rowptr_out(int32_t* dst, const int64_t* src, int64_t n, int32_t off, cudaStream_t st);
+void launch_rowptr_out(int64_t* dst, const int64_t* src, int64_t n, int64_t off, cudaStream_t st);
+// row_ptr[n] = *total (the last entry of an exclusive scan written without it)
+void launch_put_last(int64_t* row_ptr, int64_t n, const int64_t* total, cudaStream_t st);
 // dst[i] = src[i] + off (row pointers of a row piece placed after earlier pieces)
 void launch_copy_offset(int32_t* dst, const int32_t* src, int64_t n, int32_t off, cudaStream_t st);
 // nbytes (multiple of 4, <= 4096) from device memory to mapped host memory, by a kernel

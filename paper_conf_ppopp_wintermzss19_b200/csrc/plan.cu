@@ -509,10 +509,12 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
 
   // ------------------------------------------------------------ SCAN ----------
   record(p, S_SCAN, st);
-  ACS_ENSURE(p->row_ptr, sizeof(int32_t) * (A->rows + 1));
-  launch_scan_rowptr(ptr<int32_t>(p->row_count), ptr<int32_t>(p->row_ptr), A->rows, scal + 16,
-                     ptr<int64_t>(p->scan_tmp), st);
-  tl_launches += 3;
+  // int64 row pointers in plan memory (any nnz(C)); C gets int32 or int64 copies
+  ACS_ENSURE(p->row_ptr, sizeof(int64_t) * (A->rows + 1));
+  launch_scan_i32(ptr<int32_t>(p->row_count), ptr<int64_t>(p->row_ptr), A->rows, scal + 16,
+                  ptr<int64_t>(p->scan_tmp), st);
+  launch_put_last(ptr<int64_t>(p->row_ptr), A->rows, scal + 16, st);
+  tl_launches += 4;
   ACS_CUDA(cudaGetLastError());
   launch_read_back(scal + 16, p->h_scal, sizeof(int64_t), st);
   launch_read_back(p->err.p, p->h_scal + 1, sizeof(int32_t), st);
@@ -522,7 +524,6 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   const int64_t nnz = p->h_scal[0];
   const int32_t errflag = *reinterpret_cast<int32_t*>(p->h_scal + 1);
   if (errflag) return set_err(ACSPGEMM_ERR_INTERNAL, "a shared row spans more chunks than one merge block handles");
-  if (nnz >= (int64_t(1) << 31)) return set_err(ACSPGEMM_ERR_INDEX_OVERFLOW, "nnz(C) >= 2^31");
   p->nnz = nnz;
   p->info.nnz_c = nnz;
   p->info.helper_bytes = helper_bytes(p);
@@ -532,24 +533,26 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   return ACSPGEMM_OK;
 }
 
-acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t st, int32_t row_off = 0) {
+// Numeric pass into C with row pointers of type I (int32: acspgemm_csr_out, int64:
+// acspgemm_csr_out64), shifted by row_off (row pieces placed after earlier pieces).
+template <typename Out, typename I>
+acspgemm_status numeric_impl_t(acspgemm_plan p, Out* C, cudaStream_t st, I row_off) {
   if (!p->ready) return set_err(ACSPGEMM_ERR_NOT_READY, "numeric called without a successful symbolic");
   if (!C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C is NULL");
   if (p->rows > 0 && !C->row_ptr) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C.row_ptr is NULL");
   if (p->nnz > 0 && (!C->col_idx || !C->val)) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C.col_idx/val is NULL");
+  if (sizeof(I) == 4 && (int64_t)row_off + p->nnz >= (int64_t(1) << 31))
+    return set_err(ACSPGEMM_ERR_INDEX_OVERFLOW, "nnz(C) >= 2^31: int32 row_ptr (use acspgemm_numeric64)");
   const long long l0 = tl_launches;
   C->rows = p->rows;
   C->cols = p->cols;
   C->nnz = p->nnz;
   if (p->empty) {
-    if (p->rows >= 0 && C->row_ptr) {
-      ACS_CUDA(cudaMemsetAsync(C->row_ptr, 0, sizeof(int32_t) * (p->rows + 1), st));
-      launch_add_offset(C->row_ptr, p->rows + 1, row_off, st);
-    }
+    if (p->rows >= 0 && C->row_ptr) launch_rowptr_out(C->row_ptr, nullptr, p->rows + 1, row_off, st);
     p->info.kernel_launches = p->launches_sym;
     return ACSPGEMM_OK;
   }
-  launch_copy_offset(C->row_ptr, ptr<int32_t>(p->row_ptr), p->rows + 1, row_off, st);
+  launch_rowptr_out(C->row_ptr, ptr<int64_t>(p->row_ptr), p->rows + 1, row_off, st);
   tl_launches += 1;
   record(p, S_CC, st);
   CopyArgs ca;
@@ -562,7 +565,7 @@ acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t 
   ca.pool_val = p->pool_val.p;
   ca.merge_col = ptr<int32_t>(p->merge_col);
   ca.merge_val = p->merge_val.p;
-  ca.row_ptr = ptr<int32_t>(p->row_ptr);
+  ca.row_ptr = ptr<int64_t>(p->row_ptr);
   ca.c_col = C->col_idx;
   ca.c_val = C->val;
   launch_copy(ca, p->f64, st);
@@ -571,6 +574,10 @@ acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t 
   ACS_CUDA(cudaGetLastError());
   p->info.kernel_launches = p->launches_sym + (tl_launches - l0);
   return ACSPGEMM_OK;
+}
+
+acspgemm_status numeric_impl(acspgemm_plan p, acspgemm_csr_out* C, cudaStream_t st, int32_t row_off = 0) {
+  return numeric_impl_t<acspgemm_csr_out, int32_t>(p, C, st, row_off);
 }
 
 // ------------------------------------------------------------ debug kernels ------
@@ -777,6 +784,11 @@ acspgemm_status acspgemm_numeric(acspgemm_plan p, acspgemm_csr_out* C, void* str
   return numeric_impl(p, C, reinterpret_cast<cudaStream_t>(stream));
 }
 
+acspgemm_status acspgemm_numeric64(acspgemm_plan p, acspgemm_csr_out64* C, void* stream) {
+  if (!p) return set_err(ACSPGEMM_ERR_INVALID_ARG, "plan is NULL");
+  return numeric_impl_t<acspgemm_csr_out64, int64_t>(p, C, static_cast<cudaStream_t>(stream), 0);
+}
+
 acspgemm_status acspgemm_multiply(const acspgemm_csr_in* A, const acspgemm_csr_in* B, acspgemm_csr_out* C,
                                   void* stream, acspgemm_dtype dtype) {
   if (!C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "C is NULL");
@@ -786,6 +798,8 @@ acspgemm_status acspgemm_multiply(const acspgemm_csr_in* A, const acspgemm_csr_i
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   int64_t nnz = 0;
   s = acspgemm_symbolic(p, A, B, dtype, stream, &nnz);
+  if (s == ACSPGEMM_OK && nnz >= (int64_t(1) << 31))
+    s = set_err(ACSPGEMM_ERR_INDEX_OVERFLOW, "nnz(C) >= 2^31: int32 row_ptr (use acspgemm_numeric64)");
   if (s == ACSPGEMM_OK) {
     const size_t vb = dtype == ACSPGEMM_F64 ? 8 : 4;
     C->row_ptr = nullptr; C->col_idx = nullptr; C->val = nullptr;
