@@ -116,12 +116,6 @@ void launch_rowptr_out(int64_t* dst, const int64_t* src, int64_t n, int64_t off,
   k_rowptr_out<int64_t><<<grid, 256, 0, st>>>(dst, src, n, off);
 }
 
-__global__ void k_put_last(int64_t* row_ptr, int64_t n, const int64_t* total) { row_ptr[n] = *total; }
-
-void launch_put_last(int64_t* row_ptr, int64_t n, const int64_t* total, cudaStream_t st) {
-  k_put_last<<<1, 1, 0, st>>>(row_ptr, n, total);
-}
-
 __global__ void k_add_offset(int32_t* __restrict__ p, int64_t n, int32_t off) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     p[i] += off;

@@ -31,8 +31,8 @@ void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int
 int64_t scan_tmp_elems(int64_t n);
 void launch_scan_i64(const int64_t* in, int64_t* out, int64_t n, int64_t* total_dev, int64_t* tmp, cudaStream_t st);
 void launch_scan_i32(const int32_t* in, int64_t* out, int64_t n, int64_t* total_dev, int64_t* tmp, cudaStream_t st);
-// row_ptr: exclusive scan of int32 counts into int32 row_ptr[n+1] (+int64 total).
-void launch_scan_rowptr(const int32_t* in, int32_t* row_ptr, int64_t n, int64_t* total_dev, int64_t* tmp,
+// row_ptr: exclusive scan of int32 counts into int64 row_ptr[n+1] (+ the total).
+void launch_scan_rowptr(const int32_t* in, int64_t* row_ptr, int64_t n, int64_t* total_dev, int64_t* tmp,
                         cudaStream_t st);
 
 // ---- stage 2: AC-ESC (esc.cu) ---------------------------------------------------
@@ -165,8 +165,6 @@ void launch_copy(const CopyArgs& a, bool f64, cudaStream_t st);
 // src nullptr: dst[i] = off)
 void launch_rowptr_out(int32_t* dst, const int64_t* src, int64_t n, int32_t off, cudaStream_t st);
 void launch_rowptr_out(int64_t* dst, const int64_t* src, int64_t n, int64_t off, cudaStream_t st);
-// row_ptr[n] = *total (the last entry of an exclusive scan written without it)
-void launch_put_last(int64_t* row_ptr, int64_t n, const int64_t* total, cudaStream_t st);
 // dst[i] = src[i] + off (row pointers of a row piece placed after earlier pieces)
 void launch_copy_offset(int32_t* dst, const int32_t* src, int64_t n, int32_t off, cudaStream_t st);
 // nbytes (multiple of 4, <= 4096) from device memory to mapped host memory, by a kernel

@@ -511,10 +511,9 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   record(p, S_SCAN, st);
   // int64 row pointers in plan memory (any nnz(C)); C gets int32 or int64 copies
   ACS_ENSURE(p->row_ptr, sizeof(int64_t) * (A->rows + 1));
-  launch_scan_i32(ptr<int32_t>(p->row_count), ptr<int64_t>(p->row_ptr), A->rows, scal + 16,
-                  ptr<int64_t>(p->scan_tmp), st);
-  launch_put_last(ptr<int64_t>(p->row_ptr), A->rows, scal + 16, st);
-  tl_launches += 4;
+  launch_scan_rowptr(ptr<int32_t>(p->row_count), ptr<int64_t>(p->row_ptr), A->rows, scal + 16,
+                     ptr<int64_t>(p->scan_tmp), st);
+  tl_launches += 3;
   ACS_CUDA(cudaGetLastError());
   launch_read_back(scal + 16, p->h_scal, sizeof(int64_t), st);
   launch_read_back(p->err.p, p->h_scal + 1, sizeof(int32_t), st);

@@ -87,9 +87,9 @@ void launch_scan_i64(const int64_t* in, int64_t* out, int64_t n, int64_t* total_
 void launch_scan_i32(const int32_t* in, int64_t* out, int64_t n, int64_t* total_dev, int64_t* tmp, cudaStream_t st) {
   scan_impl<int32_t, int64_t>(in, out, n, total_dev, tmp, false, st);
 }
-void launch_scan_rowptr(const int32_t* in, int32_t* row_ptr, int64_t n, int64_t* total_dev, int64_t* tmp,
+void launch_scan_rowptr(const int32_t* in, int64_t* row_ptr, int64_t n, int64_t* total_dev, int64_t* tmp,
                         cudaStream_t st) {
-  scan_impl<int32_t, int32_t>(in, row_ptr, n, total_dev, tmp, true, st);
+  scan_impl<int32_t, int64_t>(in, row_ptr, n, total_dev, tmp, true, st);
 }
 
 }  // namespace acs
