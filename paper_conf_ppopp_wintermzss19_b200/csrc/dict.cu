@@ -60,12 +60,13 @@ constexpr int DICT_EPAD = 2 * DICT_W;   // entries past the last one a prefetchi
 
 // One warp's accumulator over the dictionary: acc[i] sums the current row's products of
 // dictionary column i, mark[i] = 1 when the row has column i, list = the row's indices
-// in column order while it is emitted.  Slot DICT_DMAX is the dummy of idle lanes.
+// in column order while it is emitted.  Slots DICT_DMAX + lane are the idle lanes'
+// dummies (one per lane: no two lanes of a wave ever touch one slot).
 template <typename T>
 struct DictWarp {
-  T acc[DICT_DMAX + 1];
+  T acc[DICT_DMAX + 32];
   union {                        // the marks are read into registers before the list is built
-    alignas(16) uint8_t mark[DICT_DMAX + 16];
+    alignas(16) uint8_t mark[DICT_DMAX + 32];
     uint16_t list[DICT_DMAX];
   };
 };
@@ -77,7 +78,7 @@ struct DictSmem {
   int wd[NPB + 1];               // exclusive product prefix over compacted entries
   int row_first[NPB + 1];
   int row_of[NPB];
-  uint16_t sidx[DICT_NSMAX + 32];  // dictionary index of every staged B entry; pads: DICT_DMAX
+  uint16_t sidx[DICT_NSMAX + 32];  // dictionary index of every staged B entry; pads: DICT_DMAX + lane
   int dcol[DICT_DMAX];           // dictionary index -> column
   union {
     int rp_cache[NPB + 1];
@@ -100,7 +101,7 @@ struct DictSmem {
   int scratch[40];
   int nd, cmin, cmax, bad;
 };
-static_assert(DICT_DMAX % 32 == 0, "the dummy slot lies outside the emitted windows");
+static_assert(DICT_DMAX % 32 == 0, "the dummy slots lie outside the emitted windows");
 
 // Waves of one row: wave (entry c, offset o) = B entries [o, o+32) of entry c's row.
 // Staged B rows are padded to whole waves with the dummy index, so a lane past the B row
@@ -136,8 +137,8 @@ struct DictCursor {
 };
 
 // Accumulate one batch of waves and mark their dictionary indices.  Lanes without a
-// product use the dummy slot DICT_DMAX, so every wave's read-modify-write runs converged
-// and in wave order.
+// product use their own dummy slot DICT_DMAX + lane (the staged pads hold it), so every
+// wave's read-modify-write runs converged; __syncwarp orders the waves (left fold).
 template <int W, typename T>
 __device__ __forceinline__ void dict_accumulate(DictWarp<T>& Wp, const int (&idx)[W], const T (&av)[W],
                                                 const T (&bv)[W]) {
@@ -146,6 +147,7 @@ __device__ __forceinline__ void dict_accumulate(DictWarp<T>& Wp, const int (&idx
     const T p = vmul(av[w], bv[w]);
     Wp.acc[idx[w]] = vadd(Wp.acc[idx[w]], p);
     Wp.mark[idx[w]] = 1;
+    __syncwarp();                        // wave w's writes are visible to wave w+1's lanes
   }
 }
 
@@ -256,7 +258,7 @@ __global__ void __launch_bounds__(DICT_THREADS, DICT_WARPS == 8 ? 2 : 3) k_dict(
     S.ent[nent + tid] = make_int4(0, 0, 0, 0);
     S.a_val[nent + tid] = (T)0;
   }
-  if (tid < 32) S.sidx[DICT_NSMAX + tid] = DICT_DMAX;   // the pad wave of finished rows
+  if (tid < 32) S.sidx[DICT_NSMAX + tid] = DICT_DMAX + tid;   // the pad wave of finished rows
   for (int i = tid; i < DICT_RH; i += DICT_THREADS) S.u.rh.key[i] = -1;
   if (tid == 0) { S.nd = 0; S.cmin = INT_MAX; S.cmax = INT_MIN; S.bad = 0; }
   __syncthreads();
@@ -419,7 +421,7 @@ __global__ void __launch_bounds__(DICT_THREADS, DICT_WARPS == 8 ? 2 : 3) k_dict(
       const int g = g0 + u * DICT_WARPS;
       if (g < nwaves) {
         const int c = col[u] - cmin;
-        int idx = DICT_DMAX;
+        int idx = DICT_DMAX + lane;      // pad: this lane's dummy
         if (v[u]) {
           idx = S.u.bm.pre[c >> 5] + __popc(S.u.bm.bits[c >> 5] & ((1u << (c & 31)) - 1u));
           S.dcol[idx] = col[u];
@@ -432,8 +434,8 @@ __global__ void __launch_bounds__(DICT_THREADS, DICT_WARPS == 8 ? 2 : 3) k_dict(
 
   // ---------------- rows: accumulate, emit in dictionary (= column) order ----------------
   DictWarp<T>& Wp = S.u.w[w];
-  for (int i = lane; i <= DICT_DMAX; i += 32) Wp.acc[i] = (T)(-0.0);
-  for (int i = lane; i < DICT_DMAX + 16; i += 32) Wp.mark[i] = 0;
+  for (int i = lane; i < DICT_DMAX + 32; i += 32) Wp.acc[i] = (T)(-0.0);
+  for (int i = lane; i < DICT_DMAX + 32; i += 32) Wp.mark[i] = 0;
   __syncwarp();
   const int rlo = S.wrow[w], rhi = S.wrow[w + 1];
   const int64_t wbase_pool = a.pool_off[b] + (rlo < nrows ? S.wd[S.row_first[rlo]] : 0);
