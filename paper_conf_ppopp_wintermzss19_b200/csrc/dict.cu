@@ -9,7 +9,8 @@
 // once per block instead of once per product and per row:
 //   * Distinct B rows.  The block's NPB entries reference far fewer distinct B rows
 //     (27-point stencil: ~190 for 512 entries); they are found with a small hash on the
-//     B row start and staged back to back (offsets by a block scan).
+//     B row start and staged back to back, each padded to whole waves of 32 (offsets by
+//     a block scan; pads hold a per-lane dummy index).
 //   * Dictionary.  Every column of the staged B rows sets a bit in a bitmap over the
 //     block's column span [cmin, cmax]; a prefix of the word popcounts ranks them: the
 //     dictionary index of column c is the number of distinct block columns below c.  So
@@ -22,11 +23,11 @@
 //     of a wave touch distinct slots, and waves run in order: every output is the left
 //     fold of its products in A-entry order from -0.0, exactly what the hash accumulator
 //     computes (bit-identical results; fp64 rows inside a block equal the oracle's
-//     Gustavson order bit for bit).  A per-warp bitmap over the dictionary (shared-memory
-//     atomicOr per wave) marks the row's columns.
-//   * Emission.  Lane k takes bitmap word k; a warp scan of the popcounts places every
-//     set bit, and the row's entries are written to the chunk coalesced in dictionary
-//     order = column order: already sorted.
+//     Gustavson order bit for bit).  A byte per dictionary slot marks the row's columns.
+//   * Emission.  Lane k turns the marks of dictionary window k (32 slots) into a word; a
+//     warp scan of the popcounts orders the row's indices into a list, and the row's
+//     entries are written to the chunk coalesced in dictionary order = column order:
+//     already sorted.
 // A block whose distinct B rows hold more than DICT_NSMAX entries, whose span exceeds
 // DICT_SPAN columns or whose dictionary exceeds DICT_DMAX columns is left to k_hash
 // (hash_done stays 1; the test depends only on the data, so the choice is
