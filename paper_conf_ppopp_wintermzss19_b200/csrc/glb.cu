@@ -134,11 +134,21 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
     const int64_t nzb = s_nz[s] + (b - s_base[s]) * NPB;
     const int64_t nze = min(nzb + (int64_t)NPB, s_nz[s + 1]);
     int64_t sum = 0, waves = 0;
-    for (int64_t p = nzb + lane; p < nze; p += 32) {
-      const int k = acol[p];
-      const int len = brp[k + 1] - brp[k];
-      sum += len;
-      waves += (len + 31) >> 5;
+    // all of the block's column loads first (NPB / 32 per lane), then the B row gathers
+    constexpr int PER_LANE = NPB / 32;
+    int k[PER_LANE];
+#pragma unroll
+    for (int j = 0; j < PER_LANE; ++j) {
+      const int64_t p = nzb + lane + 32 * j;
+      k[j] = p < nze ? acol[p] : -1;
+    }
+#pragma unroll
+    for (int j = 0; j < PER_LANE; ++j) {
+      if (k[j] >= 0) {
+        const int len = brp[k[j] + 1] - brp[k[j]];
+        sum += len;
+        waves += (len + 31) >> 5;
+      }
     }
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) {
