@@ -159,6 +159,19 @@ acspgemm_status acspgemm_symbolic(acspgemm_plan plan, const acspgemm_csr_in* A, 
  * ACSPGEMM_ERR_INDEX_OVERFLOW when nnz(C) >= 2^31 (int32 row_ptr): use acspgemm_numeric64. */
 acspgemm_status acspgemm_numeric(acspgemm_plan plan, acspgemm_csr_out* C, void* stream);
 
+/* Re-multiply with new VALUES on the pattern of the plan's last acspgemm_symbolic (SURVEY
+ * §8(f)-2, e.g. an AMG hierarchy re-setup): A and B must have exactly the structure
+ * (row_ptr, col_idx contents, dimensions, dtype) of that call -- the caller guarantees it,
+ * the library checks only the dimensions -- and C is caller-allocated with the nnz that
+ * call returned.  Produces the same bits as a fresh symbolic + numeric on the new values.
+ * No host synchronisation: the sizes the symbolic read back are replayed, and the whole
+ * launch sequence is captured once into a CUDA graph (re-captured when any pointer
+ * changes; on the legacy default stream it runs uncaptured).  Asynchronous on `stream`.
+ * Any later acspgemm_symbolic on the plan starts a new pattern.  Stage times are not
+ * collected by this call. */
+acspgemm_status acspgemm_numeric_update(acspgemm_plan plan, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
+                                        acspgemm_csr_out* C, void* stream);
+
 /* Numeric pass into a C with int64 row_ptr[rows+1] (any nnz(C); outputs
  * beyond 2^31 entries, e.g. skewed graph products).  Otherwise as acspgemm_numeric. */
 acspgemm_status acspgemm_numeric64(acspgemm_plan plan, acspgemm_csr_out64* C, void* stream);

@@ -57,6 +57,8 @@ SIGNATURES = {
     "acspgemm_symbolic": (ctypes.c_int, [VP, ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.c_int, VP, PI64]),
     "acspgemm_numeric": (ctypes.c_int, [VP, ctypes.POINTER(CsrOut), VP]),
     "acspgemm_numeric64": (ctypes.c_int, [VP, ctypes.POINTER(CsrOut64), VP]),
+    "acspgemm_numeric_update": (ctypes.c_int, [VP, ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn),
+                                               ctypes.POINTER(CsrOut), VP]),
     "acspgemm_multiply": (ctypes.c_int, [ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.POINTER(CsrOut), VP,
                                          ctypes.c_int]),
     "acspgemm_multiply_host": (ctypes.c_int, [VP, ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.c_int, VP,

@@ -168,6 +168,18 @@ class Plan:
         self.numeric(rp, col, val, stream)
         return DeviceCSR(rows, B.cols, rp, col[:nnz], val[:nnz])
 
+    def numeric_update(self, A: DeviceCSR, B: DeviceCSR, C: DeviceCSR, stream=None) -> DeviceCSR:
+        """Recompute C's values for new values of A and B on the pattern of this plan's last
+        multiply (same structure, same dtype; C from that multiply, int32 row_ptr).
+        Sync-free: replays the recorded sizes inside a CUDA graph (acspgemm_numeric_update)."""
+        if C.row_ptr.dtype != torch.int32:
+            raise TypeError("numeric_update writes an int32 row_ptr")
+        a, b = _csr_in(A), _csr_in(B)
+        c = CsrOut(0, 0, 0, C.row_ptr.data_ptr(), C.col.data_ptr(), C.val.data_ptr())
+        check(self._lib.acspgemm_numeric_update(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c),
+                                                _stream_ptr(stream)), "acspgemm_numeric_update")
+        return C
+
     def multiply_host(self, A, B, out=None, pieces: int = 4, stream=None):
         """End to end through acspgemm_multiply_host: A and B on the host (objects with
         rows, cols, row_ptr, col, val as numpy arrays or CPU tensors; int32 indices),

@@ -16,6 +16,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <vector>
 
 #include <algorithm>
 
@@ -92,6 +93,16 @@ struct acspgemm_plan_s {
   acspgemm_info info;
   long long launches_sym = 0;
   int dev = 0;
+  // pattern replay (acspgemm_numeric_update): the host values of every read-back of the
+  // last symbolic, in order, and the problem they describe; replaying them makes the
+  // launch sequence sync-free, so it is captured once into a CUDA graph
+  std::vector<std::vector<int64_t>> rec;
+  size_t rec_pos = 0;
+  bool replay = false;
+  int64_t rec_dims[6] = {-1, -1, -1, -1, -1, -1};   // A rows, cols, nnz; B rows, cols, nnz
+  int rec_dtype = -1;
+  cudaGraphExec_t gexec = nullptr;
+  const void* gkey[9] = {};
 };
 
 namespace {
@@ -133,7 +144,7 @@ void free_buf(DevBuf& b) {
 }
 
 void record(acspgemm_plan p, int stage, cudaStream_t st) {
-  if (p->opt.collect_stage_times && p->ev_ok) cudaEventRecord(p->ev[stage], st);
+  if (p->opt.collect_stage_times && p->ev_ok && !p->replay) cudaEventRecord(p->ev[stage], st);
 }
 
 acspgemm_status check_in(const acspgemm_csr_in* M, const char* name) {
@@ -159,10 +170,20 @@ int64_t helper_bytes(acspgemm_plan p) {
   return t;
 }
 
+// Read n device words into h_scal (a host round trip), recorded for pattern replay; in
+// replay the recorded values are used instead (no launch, no synchronisation).
 acspgemm_status sync_read(acspgemm_plan p, const int64_t* dev, int n, cudaStream_t st) {
+  if (p->replay) {
+    if (p->rec_pos >= p->rec.size() || (int)p->rec[p->rec_pos].size() != n)
+      return set_err(ACSPGEMM_ERR_INTERNAL, "pattern replay out of step");
+    std::memcpy(p->h_scal, p->rec[p->rec_pos].data(), sizeof(int64_t) * n);
+    ++p->rec_pos;
+    return ACSPGEMM_OK;
+  }
   launch_read_back(dev, p->h_scal, (int)sizeof(int64_t) * n, st);
   tl_launches += 1;
   ACS_CUDA(cudaStreamSynchronize(st));
+  p->rec.emplace_back(p->h_scal, p->h_scal + n);
   return ACSPGEMM_OK;
 }
 
@@ -178,6 +199,15 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   if (A->cols != B->rows) return set_err(ACSPGEMM_ERR_DIM_MISMATCH, "A.cols != B.rows");
   ACS_CUDA(cudaGetDevice(&p->dev));
   const long long l0 = tl_launches;
+  if (p->replay) {
+    p->rec_pos = 0;
+  } else {
+    p->rec.clear();
+    if (p->gexec) { cudaGraphExecDestroy(p->gexec); p->gexec = nullptr; }
+    const int64_t dims[6] = {A->rows, A->cols, A->nnz, B->rows, B->cols, B->nnz};
+    std::memcpy(p->rec_dims, dims, sizeof(dims));
+    p->rec_dtype = (int)dtype;
+  }
   p->ready = false;
   p->f64 = dtype == ACSPGEMM_F64;
   p->rows = A->rows;
@@ -205,7 +235,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   int64_t* scal = ptr<int64_t>(p->scal);
   ACS_CUDA(cudaMemsetAsync(p->err.p, 0, sizeof(int32_t) * 4, st));
 
-  if (p->opt.validate_inputs) {
+  if (p->opt.validate_inputs && !p->replay) {
     launch_validate(Av, ptr<int32_t>(p->err), st);
     launch_validate(Bv, ptr<int32_t>(p->err), st);
     tl_launches += 2;
@@ -266,9 +296,11 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   k_put_i64<<<1, 1, 0, st>>>(scal + 2, nblocks_dev);
   tl_launches += 1;
   ACS_CUDA(cudaGetLastError());
-  // segment boundaries (for info) ride along with the first read-back
-  launch_read_back(p->seg.p, p->h_scal + H_SEG_INFO, (int)sizeof(int64_t) * (nseg + 1), st);
-  tl_launches += 1;
+  // segment boundaries (for info) ride along with the first read-back (replay: unchanged)
+  if (!p->replay) {
+    launch_read_back(p->seg.p, p->h_scal + H_SEG_INFO, (int)sizeof(int64_t) * (nseg + 1), st);
+    tl_launches += 1;
+  }
   if ((s = sync_read(p, scal, 4, st)) != ACSPGEMM_OK) return s;
   const int64_t products = p->h_scal[0], slots = p->h_scal[1], nblocks = p->h_scal[2], ncand = p->h_scal[3];
   p->info.products = products;
@@ -515,13 +547,24 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
                      ptr<int64_t>(p->scan_tmp), st);
   tl_launches += 3;
   ACS_CUDA(cudaGetLastError());
-  launch_read_back(scal + 16, p->h_scal, sizeof(int64_t), st);
-  launch_read_back(p->err.p, p->h_scal + 1, sizeof(int32_t), st);
-  tl_launches += 2;
   record(p, S_CC, st);
-  ACS_CUDA(cudaStreamSynchronize(st));
-  const int64_t nnz = p->h_scal[0];
-  const int32_t errflag = *reinterpret_cast<int32_t*>(p->h_scal + 1);
+  int64_t nnz;
+  int32_t errflag;
+  if (p->replay) {
+    if (p->rec_pos >= p->rec.size() || p->rec[p->rec_pos].size() != 2)
+      return set_err(ACSPGEMM_ERR_INTERNAL, "pattern replay out of step");
+    nnz = p->rec[p->rec_pos][0];
+    errflag = (int32_t)p->rec[p->rec_pos][1];
+    ++p->rec_pos;
+  } else {
+    launch_read_back(scal + 16, p->h_scal, sizeof(int64_t), st);
+    launch_read_back(p->err.p, p->h_scal + 1, sizeof(int32_t), st);
+    tl_launches += 2;
+    ACS_CUDA(cudaStreamSynchronize(st));
+    nnz = p->h_scal[0];
+    errflag = *reinterpret_cast<int32_t*>(p->h_scal + 1);
+    p->rec.push_back({nnz, (int64_t)errflag});
+  }
   if (errflag) return set_err(ACSPGEMM_ERR_INTERNAL, "a shared row spans more chunks than one merge block handles");
   p->nnz = nnz;
   p->info.nnz_c = nnz;
@@ -724,8 +767,10 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
                   &p->scan_tmp, &p->kflag, &p->kpos, &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan,
                   &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
                   &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->lgiant, &p->g_lo, &p->g_nsl,
-                  &p->g_base, &p->g_tcol, &p->g_tval, &p->g_tcnt};
+                  &p->g_base, &p->g_tcol, &p->g_tval, &p->g_tcnt, &p->hdone, &p->esc_list,
+                  &p->esc_list_small};
   for (DevBuf* b : bs) free_buf(*b);
+  if (p->gexec) cudaGraphExecDestroy(p->gexec);
   for (int i = 0; i < 3; ++i) {
     free_buf(p->hp_a[i]);
     free_buf(p->hp_b[i]);
@@ -781,6 +826,54 @@ acspgemm_status acspgemm_symbolic(acspgemm_plan p, const acspgemm_csr_in* A, con
 acspgemm_status acspgemm_numeric(acspgemm_plan p, acspgemm_csr_out* C, void* stream) {
   if (!p) return set_err(ACSPGEMM_ERR_INVALID_ARG, "plan is NULL");
   return numeric_impl(p, C, reinterpret_cast<cudaStream_t>(stream));
+}
+
+acspgemm_status acspgemm_numeric_update(acspgemm_plan p, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
+                                        acspgemm_csr_out* C, void* stream) {
+  if (!p || !A || !B || !C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
+  if (!p->ready || p->rec_dtype < 0)
+    return set_err(ACSPGEMM_ERR_NOT_READY, "numeric_update needs a successful symbolic of the same pattern");
+  const int64_t dims[6] = {A->rows, A->cols, A->nnz, B->rows, B->cols, B->nnz};
+  if (std::memcmp(dims, p->rec_dims, sizeof(dims)) != 0)
+    return set_err(ACSPGEMM_ERR_INVALID_ARG, "numeric_update: A/B dimensions differ from the last symbolic");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const acspgemm_dtype dtype = (acspgemm_dtype)p->rec_dtype;
+  if (p->empty) {                        // no entries: only the row pointers
+    int64_t nnz = 0;
+    acspgemm_status s = symbolic_impl(p, A, B, dtype, st, &nnz);
+    return s == ACSPGEMM_OK ? numeric_impl(p, C, st) : s;
+  }
+  const void* key[9] = {A->row_ptr, A->col_idx, A->val, B->row_ptr, B->col_idx, B->val,
+                        C->row_ptr, C->col_idx, C->val};
+  if (p->gexec && std::memcmp(key, p->gkey, sizeof(key)) == 0) {
+    ACS_CUDA(cudaGraphLaunch(p->gexec, st));
+    return ACSPGEMM_OK;
+  }
+  if (p->gexec) { cudaGraphExecDestroy(p->gexec); p->gexec = nullptr; }
+  // the legacy default stream cannot be captured: replay without a graph (still sync-free)
+  const bool capture = st != nullptr && st != cudaStreamLegacy && st != cudaStreamPerThread;
+  cudaGraph_t g = nullptr;
+  if (capture) ACS_CUDA(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed));
+  p->replay = true;
+  int64_t nnz = 0;
+  acspgemm_status s = symbolic_impl(p, A, B, dtype, st, &nnz);
+  if (s == ACSPGEMM_OK) s = numeric_impl(p, C, st);
+  p->replay = false;
+  if (capture) {
+    const cudaError_t e = cudaStreamEndCapture(st, &g);
+    if (s == ACSPGEMM_OK && e != cudaSuccess) s = set_err(ACSPGEMM_ERR_CUDA, cudaGetErrorString(e));
+    if (s == ACSPGEMM_OK) {
+      const cudaError_t ei = cudaGraphInstantiate(&p->gexec, g, 0);
+      if (ei != cudaSuccess) { p->gexec = nullptr; s = set_err(ACSPGEMM_ERR_CUDA, cudaGetErrorString(ei)); }
+    }
+    if (g) cudaGraphDestroy(g);
+    if (s == ACSPGEMM_OK) {
+      std::memcpy(p->gkey, key, sizeof(key));
+      const cudaError_t el = cudaGraphLaunch(p->gexec, st);
+      if (el != cudaSuccess) s = set_err(ACSPGEMM_ERR_CUDA, cudaGetErrorString(el));
+    }
+  }
+  return s;
 }
 
 acspgemm_status acspgemm_numeric64(acspgemm_plan p, acspgemm_csr_out64* C, void* stream) {
