@@ -123,6 +123,7 @@ typedef struct {
   int64_t segment_rows[65];
   int64_t nhash_blocks;      /* blocks completed by an accumulator (dictionary or hash; R33, R31) */
   int64_t ndict_blocks;      /* of them, blocks completed by the column-dictionary accumulator (R33) */
+  int64_t nrow_blocks;       /* blocks completed by the per-row accumulator for short rows (R34) */
 } acspgemm_info;
 
 /* Defaults: no pool limit, no validation, no stage times, 8 segments, adaptive strategy. */

@@ -44,7 +44,7 @@ class Info(ctypes.Structure):
                 ("nsearch", I64), ("nmulti_groups", I64), ("merge_elems", I64),
                 ("pool_bytes", I64), ("helper_bytes", I64), ("pool_estimate_bytes", ctypes.c_double),
                 ("kernel_launches", I64), ("nsegments", I32), ("segment_rows", I64 * 65),
-                ("nhash_blocks", I64), ("ndict_blocks", I64)]
+                ("nhash_blocks", I64), ("ndict_blocks", I64), ("nrow_blocks", I64)]
 
 
 # name -> (restype, argtypes); every symbol include/acspgemm.h declares

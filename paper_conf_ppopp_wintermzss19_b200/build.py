@@ -16,7 +16,7 @@ CSRC = os.path.join(HERE, "csrc")
 _TAG = os.environ.get("ACS_BUILD_TAG", "")
 BUILD = os.path.join(HERE, "build" + (f"_{_TAG}" if _TAG else ""))
 SO = os.path.join(HERE, "libacspgemm" + (f"_{_TAG}" if _TAG else "") + ".so")
-SOURCES = ["glb.cu", "scan.cu", "esc.cu", "esc_small.cu", "hash.cu", "dict.cu", "merge.cu", "copy.cu", "plan.cu"]
+SOURCES = ["glb.cu", "scan.cu", "esc.cu", "esc_small.cu", "hash.cu", "dict.cu", "rows.cu", "merge.cu", "copy.cu", "plan.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr", "-ftz=false", "-prec-div=true",

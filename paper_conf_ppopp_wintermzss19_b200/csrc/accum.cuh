@@ -65,26 +65,34 @@ __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cac
   const int64_t rowsA = a.A.rows;
   constexpr int NPT = NPB / NT;          // A entries per thread (blocked)
   static_assert(NPB % NT == 0, "NPB must be a multiple of NT");
-  for (int t = tid; t <= NPB; t += NT) {
-    const int64_t r = (int64_t)r0 + t;
-    rp_cache[t] = r <= rowsA ? arp[r] : INT_MAX;
-  }
-  __syncthreads();
+  // the entries' loads and their B row gathers are issued before the row pointers'
+  // barrier, so the two chains of global loads overlap
   int len[NPT], row[NPT], bst[NPT];
   T av[NPT];
 #pragma unroll
   for (int j = 0; j < NPT; ++j) {
     const int e = tid * NPT + j;
     len[j] = 0;
-    row[j] = INT_MAX;
     bst[j] = 0;
     av[j] = (T)0;
     if (e < n_a) {
-      const int nz = nzb + e;
-      const int k = acol[nz];
-      av[j] = aval[nz];
+      const int k = acol[nzb + e];
+      av[j] = aval[nzb + e];
       bst[j] = brp[k];
       len[j] = brp[k + 1] - bst[j];
+    }
+  }
+  for (int t = tid; t <= NPB; t += NT) {
+    const int64_t r = (int64_t)r0 + t;
+    rp_cache[t] = r <= rowsA ? arp[r] : INT_MAX;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < NPT; ++j) {
+    const int e = tid * NPT + j;
+    row[j] = INT_MAX;
+    if (e < n_a) {
+      const int nz = nzb + e;
       int r;
       if (nz < rp_cache[NPB]) {
         int lo = 0, hi = NPB - 1;
@@ -165,9 +173,10 @@ __device__ __forceinline__ void split_rows(const int* wd, const int* row_first, 
 }
 
 // One chunk descriptor per warp that emitted rows (L424-L428), in warp order = row
-// order; wout[q] = {count, first_row, last_row, first_count, last_count}.  Thread 0.
+// order; wout[q] = {count, first_row, last_row, first_count, last_count}; counts the
+// block in *counter (info only).  Thread 0.
 __device__ __forceinline__ void emit_warp_chunks(const EscArgs& a, int b, int nw, const int* wrow, const int (*wout)[5],
-                                                 const int* wd, const int* row_first) {
+                                                 const int* wd, const int* row_first, int64_t* counter) {
   const int64_t pool_base = a.pool_off[b];
   const int64_t desc_base = a.desc_off[b];
   int seq = 0, used = 0;
@@ -187,7 +196,7 @@ __device__ __forceinline__ void emit_warp_chunks(const EscArgs& a, int b, int nw
   }
   a.nchunks[b] = seq;
   a.used[b] = used;
-  atomicAdd(reinterpret_cast<unsigned long long*>(a.hash_count), 1ull);
+  atomicAdd(reinterpret_cast<unsigned long long*>(counter), 1ull);
 }
 
 }  // namespace acs

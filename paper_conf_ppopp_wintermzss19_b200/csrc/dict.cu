@@ -501,7 +501,7 @@ __global__ void __launch_bounds__(DICT_THREADS, DICT_WARPS == 8 ? 2 : 3) k_dict(
   }
   __syncthreads();
   if (tid == 0) {
-    emit_warp_chunks(a, b, DICT_WARPS, S.wrow, S.wout, S.wd, S.row_first);
+    emit_warp_chunks(a, b, DICT_WARPS, S.wrow, S.wout, S.wd, S.row_first, a.hash_count);
     a.hash_done[b] = 2;
     atomicAdd(reinterpret_cast<unsigned long long*>(a.dict_count), 1ull);
   }

@@ -51,9 +51,10 @@ struct EscArgs {
   int32_t* used;                // per block: chunk elements written
   int32_t* row_count;           // per row of C
   int32_t* hash_done;           // per block: in: 1 = hash candidate (k_block_bounds); out: 2 = finished
-                                // by k_dict, 1 = finished by k_hash, 0 = AC-ESC (nullptr: none)
+                                // by k_dict, 1 = by k_hash, 3 = by k_rows, 0 = AC-ESC (nullptr: none)
   int64_t* hash_count;          // blocks finished by k_dict or k_hash (atomic counter, info only)
   int64_t* dict_count;          // blocks finished by k_dict (atomic counter, info only)
+  int64_t* rows_count;          // blocks finished by k_rows (atomic counter, info only)
   int32_t* esc_list;            // adaptive: blocks left to AC-ESC [nblocks]
   int64_t* esc_count;           // adaptive: their number (zeroed before launch_hash)
   int64_t* esc_next;            // adaptive: grab counter of the persistent k_esc (zeroed)
@@ -70,6 +71,9 @@ void launch_hash(const EscArgs& a, bool f64, cudaStream_t st);
 // column-dictionary accumulator (dict.cu, reading R33): runs before launch_hash on the
 // same stream; blocks it finishes get hash_done = 2, the rest stay hash candidates
 void launch_dict(const EscArgs& a, bool f64, cudaStream_t st);
+// per-row accumulator for blocks of short rows (rows.cu, reading R34): after launch_hash,
+// on the blocks no accumulator finished; the ones it finishes get hash_done = 3
+void launch_rows(const EscArgs& a, bool f64, cudaStream_t st);
 
 // ---- stage 3: chunk ordering, shared rows, merges (merge.cu) --------------------
 struct MergeState {

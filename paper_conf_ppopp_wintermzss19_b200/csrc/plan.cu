@@ -340,10 +340,12 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.hash_done = nullptr;
   ea.hash_count = scal + 6;
   ea.dict_count = scal + 7;
+  ea.rows_count = scal + 2;              // free after the first read-back
   ea.esc_list = ptr<int32_t>(p->esc_list);
   ea.esc_count = scal + 28;
   ea.esc_next = scal + 29;
   ACS_CUDA(cudaMemsetAsync(scal + 6, 0, 2 * sizeof(int64_t), st));
+  ACS_CUDA(cudaMemsetAsync(scal + 2, 0, sizeof(int64_t), st));
   ACS_CUDA(cudaMemsetAsync(scal + 28, 0, 2 * sizeof(int64_t), st));
   ea.blk_products = ptr<int64_t>(p->bprod);
   ea.esc_list_small = nullptr;
@@ -371,6 +373,10 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     tl_launches += nblocks > 0 ? 1 : 0;
   }
   record(p, S_HASHEND, st);
+  if (ea.hash_done) {
+    launch_rows(ea, p->f64, st);         // blocks of short rows (reading R34)
+    tl_launches += nblocks > 0 ? 1 : 0;
+  }
   if (ea.hash_done) {
     launch_esc_lists(ea, st);
     acs_launch_esc_small(&ea, p->f64, st);
@@ -407,15 +413,16 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   launch_find_shared(ms, scal + 4, st);
   tl_launches += 1 + (slots > 0 ? 5 : 0);
   ACS_CUDA(cudaGetLastError());
-  if ((s = sync_read(p, scal + 3, 5, st)) != ACSPGEMM_OK) return s;
-  p->info.nhash_blocks = p->h_scal[3];
-  p->info.ndict_blocks = p->h_scal[4];
-  p->total_chunks = p->h_scal[0];
-  p->nshared = p->h_scal[1];
+  if ((s = sync_read(p, scal + 2, 6, st)) != ACSPGEMM_OK) return s;
+  p->info.nrow_blocks = p->h_scal[0];
+  p->info.nhash_blocks = p->h_scal[4];
+  p->info.ndict_blocks = p->h_scal[5];
+  p->total_chunks = p->h_scal[1];
+  p->nshared = p->h_scal[2];
   p->max_chunks = slots;
   p->info.nchunks = p->total_chunks;
   p->info.nshared = p->nshared;
-  p->info.chunk_elems = p->h_scal[2];
+  p->info.chunk_elems = p->h_scal[3];
   const int64_t nsh = p->nshared;
   int64_t nmulti = 0, npath = 0, nsearch = 0, npair = 0, merge_total = 0, ngroups = 0, ngiant = 0;
   if (nsh > 0) {

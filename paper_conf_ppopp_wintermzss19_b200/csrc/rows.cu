@@ -1,0 +1,196 @@
+// Stage 2, adaptive alternative — per-row accumulation for blocks of short rows
+// (reading R34).
+//
+// PAPER.md L850 (§5): "choose between alternative approaches (ESC, hashing, merging)
+// depending on the load currently seen by the work distribution".  Blocks whose rows
+// each hold only a few products and columns (AMG prolongation A·P: 7 products, <= 4
+// columns per row; the Galerkin product R·(A·P): <= 32 products, 7 columns) sort a tile
+// of 512 products in AC-ESC (R32) to find them.  Here one LANE owns one row:
+//   * it walks the row's products in expansion order (A entries in storage order, each
+//     B row in order) and accumulates a_ik * b_kj into a private list of <= ROWS_LMAX
+//     (column, value) slots in shared memory (column-major over the CTA's lanes, so the
+//     lanes of a warp touch consecutive banks): a column seen before is added to its
+//     slot, a new column takes the next slot with the product itself (= -0.0 + product,
+//     the identity start of the other accumulators).  Every output is therefore the left
+//     fold of its products in A-entry order -- Gustavson's order, the same bits as the
+//     hash and dictionary accumulators (R31, R33);
+//   * the list is insertion-sorted by column and written to the warp's chunk; a warp
+//     owns a contiguous run of the block's rows and takes them 32 at a time, lane order
+//     = row order, so the chunk holds its rows in order (L424-L428).
+// Blocks with a row of more than ROWS_PMAX products are not taken; a row reaching more
+// than ROWS_LMAX distinct columns abandons the block (both tests depend only on the
+// data: the choice is deterministic).  Such blocks stay with AC-ESC.  hash_done[b] = 3
+// marks a block finished here.
+#include "accum.cuh"
+
+namespace acs {
+
+constexpr int ROWS_WARPS = THREADS / 32;
+#ifndef ACS_ROWS_LMAX
+#define ACS_ROWS_LMAX 8
+#endif
+constexpr int ROWS_LMAX = ACS_ROWS_LMAX;  // distinct columns of one row (per-lane list; 8 keeps
+                                          // shared memory at 26 KB: 8 CTAs per SM, cfg4a A·P
+                                          // 5.4 -> 4.2 ms against 16 slots)
+constexpr int ROWS_PMAX = 256;           // products of one row
+constexpr int ROWS_U = 8;                // products per lane with their B loads in flight
+
+template <typename T>
+struct RowsSmem {
+  T a_val[NPB];
+  int2 ent[NPB];                 // (B row start, length) per nonempty entry (fetch_block)
+  int wd[NPB + 1];
+  int row_first[NPB + 1];
+  int row_of[NPB];
+  union {
+    int rp_cache[NPB + 1];
+    struct {
+      int col[ROWS_LMAX][THREADS];   // lane tid's slot j at [j][tid]
+      T val[ROWS_LMAX][THREADS];
+    } l;
+  } u;
+  int wrow[ROWS_WARPS + 1];
+  int wout[ROWS_WARPS][5];
+  int scratch[40];
+  int flag;
+};
+
+template <typename T>
+__global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  RowsSmem<T>& S = *reinterpret_cast<RowsSmem<T>*>(smem_raw);
+  const unsigned FULL = 0xffffffffu;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const int b = blockIdx.x;
+  if (a.hash_done[b] != 0) return;       // finished by an accumulator already
+  const int32_t* __restrict__ bcol = a.B.col;
+  const T* __restrict__ bval = reinterpret_cast<const T*>(a.B.val);
+  if (tid == 0) S.flag = 0;
+  int nrows, nent, total;
+  fetch_block<T, int2, THREADS>(a, b, S.u.rp_cache, S.row_of, S.row_first, S.ent, S.a_val, S.wd, S.scratch, nrows,
+                                nent, total);
+  bool big = false;
+  for (int r = tid; r < nrows; r += THREADS) big |= S.wd[S.row_first[r + 1]] - S.wd[S.row_first[r]] > ROWS_PMAX;
+  if (__syncthreads_or(big)) return;     // a long row: AC-ESC
+  split_rows<ROWS_WARPS>(S.wd, S.row_first, nrows, total, S.wrow);
+  __syncthreads();
+  const int rlo = S.wrow[w], rhi = S.wrow[w + 1];
+  const int64_t wbase = a.pool_off[b] + (rlo < nrows ? S.wd[S.row_first[rlo]] : 0);
+  T* pval = reinterpret_cast<T*>(a.pool_val);
+  int32_t* pcol = a.pool_col;
+  int(*lc)[THREADS] = S.u.l.col;
+  T(*lv)[THREADS] = S.u.l.val;
+  int out = 0, first_row = -1, last_row = -1, first_count = 0, last_count = 0;
+  for (int r0 = rlo; r0 < rhi; r0 += 32) {
+    if (atomicOr(&S.flag, 0)) break;   // another warp abandoned the block (atomic: no race)
+    const int r = r0 + lane;
+    int cnt = 0;
+    bool over = false;
+    if (r < rhi) {
+      // products in expansion order, ROWS_U at a time: their B loads are all in flight
+      // before the first one is accumulated
+      int c = S.row_first[r];
+      const int c1 = S.row_first[r + 1];
+      int q = 0, qe = 0;
+      T av = (T)0;
+      if (c < c1) { const int2 e = S.ent[c]; q = e.x; qe = e.x + e.y; av = S.a_val[c]; }
+      while (c < c1) {
+        int col[ROWS_U];
+        T v[ROWS_U];
+        int n = 0;
+#pragma unroll
+        for (int u = 0; u < ROWS_U; ++u) {
+          if (c < c1) {
+            col[u] = __ldg(bcol + q);
+            v[u] = vmul(av, __ldg(bval + q));
+            n = u + 1;
+            if (++q == qe && ++c < c1) { const int2 e = S.ent[c]; q = e.x; qe = e.x + e.y; av = S.a_val[c]; }
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < ROWS_U; ++u) {
+          if (u < n) {
+            int j = 0;
+            while (j < cnt && lc[j][tid] != col[u]) ++j;
+            if (j < cnt) {
+              lv[j][tid] = vadd(lv[j][tid], v[u]);
+            } else if (cnt < ROWS_LMAX) {
+              lc[cnt][tid] = col[u];
+              lv[cnt][tid] = v[u];
+              ++cnt;
+            } else {
+              over = true;
+            }
+          }
+        }
+      }
+      // insertion sort of the row's columns (equal columns do not occur)
+      for (int i = 1; i < cnt; ++i) {
+        const int kc = lc[i][tid];
+        const T kv = lv[i][tid];
+        int j = i - 1;
+        while (j >= 0 && lc[j][tid] > kc) {
+          lc[j + 1][tid] = lc[j][tid];
+          lv[j + 1][tid] = lv[j][tid];
+          --j;
+        }
+        lc[j + 1][tid] = kc;
+        lv[j + 1][tid] = kv;
+      }
+    }
+    if (__any_sync(FULL, over)) {        // uniform per warp; the block goes to AC-ESC
+      if (lane == 0) atomicExch(&S.flag, 1);
+      break;
+    }
+    int inc = cnt;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int y = __shfl_up_sync(FULL, inc, d);
+      if (lane >= d) inc += y;
+    }
+    const int tot = __shfl_sync(FULL, inc, 31);
+    const int64_t dst = wbase + out + (inc - cnt);
+    for (int i = 0; i < cnt; ++i) {
+      pcol[dst + i] = lc[i][tid];
+      pval[dst + i] = lv[i][tid];
+    }
+    const int grow = r < rhi ? S.row_of[r] : -1;
+    if (cnt > 0) a.row_count[grow] = cnt;          // per-row counter (L362)
+    const unsigned m = __ballot_sync(FULL, cnt > 0);
+    if (m) {
+      const int fl = __ffs(m) - 1, ll = 31 - __clz(m);
+      const int frow = __shfl_sync(FULL, grow, fl), fcnt = __shfl_sync(FULL, cnt, fl);
+      const int lrow = __shfl_sync(FULL, grow, ll), lcnt = __shfl_sync(FULL, cnt, ll);
+      if (first_row < 0) { first_row = frow; first_count = fcnt; }
+      last_row = lrow;
+      last_count = lcnt;
+    }
+    out += tot;
+  }
+  if (lane == 0) {
+    S.wout[w][0] = out;
+    S.wout[w][1] = first_row;
+    S.wout[w][2] = last_row;
+    S.wout[w][3] = first_count;
+    S.wout[w][4] = last_count;
+  }
+  __syncthreads();
+  if (tid == 0 && !S.flag) {
+    emit_warp_chunks(a, b, ROWS_WARPS, S.wrow, S.wout, S.wd, S.row_first, a.rows_count);
+    a.hash_done[b] = 3;
+  }
+}
+
+template <typename T>
+static void launch_rows_t(const EscArgs& a, cudaStream_t st) {
+  const size_t smem = sizeof(RowsSmem<T>);
+  cudaFuncSetAttribute(k_rows<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k_rows<T><<<a.nblocks, THREADS, smem, st>>>(a);
+}
+
+void launch_rows(const EscArgs& a, bool f64, cudaStream_t st) {
+  if (a.nblocks <= 0) return;
+  if (f64) launch_rows_t<double>(a, st); else launch_rows_t<float>(a, st);
+}
+
+}  // namespace acs
