@@ -27,4 +27,11 @@ for cfg in [c for c in CFGS if c != "cfg4"]:
 if "cfg4" not in CFGS: sys.exit(0)
 A = poisson3d_7pt(256); P = aggregation_prolongator(256)
 run("cfg4a A*P", A, P, np.float64)
-import oracle
+# cfg4b: R·(AP) with AP from the GPU (integer values: exact), R = P^T
+from synth import CSR
+dA = acs.DeviceCSR.from_host(A, "cuda"); dP = acs.DeviceCSR.from_host(P, "cuda")
+AP = acs.Plan().multiply(dA, dP)
+rp, col, val = AP.to_numpy()
+del AP, dA, dP
+torch.cuda.empty_cache()
+run("cfg4b R*AP", transpose(P), CSR(A.rows, P.cols, rp, col, val), np.float64)
