@@ -199,6 +199,22 @@ acspgemm_status acspgemm_multiply_host(acspgemm_plan plan, const acspgemm_csr_in
                                        const acspgemm_csr_in* B_host, acspgemm_dtype dtype, void* stream,
                                        int npieces, acspgemm_csr_out* C_host, int64_t capacity);
 
+/* C = A·B within the plan's pool_limit_bytes (the paper restarts a
+ * kernel when its chunk pool runs out, L254, L844).  A and B are device CSR.  Instead of
+ * failing with OUT_OF_MEMORY when the exact pool bound exceeds the budget, the multiply
+ * runs in pieces of whole canonical segments: each piece is the longest run of
+ * segments whose bound fits (a piece over budget is retried on half as many segments --
+ * a "restart", which costs only the global load balancing of the refused piece).  Every
+ * block, chunk and merge is that of the one-piece multiply, so C is bit-identical to
+ * it.  C is allocated like acspgemm_multiply (cudaMallocAsync on `stream`, free with
+ * acspgemm_free_csr); the pieces are concatenated into it (their buffers are plan
+ * memory, kept for the next call).  *npieces / *nrestarts
+ * (nullable) receive the piece and restart counts.  A single segment over budget
+ * returns OUT_OF_MEMORY.  Synchronises `stream`; the plan's segment setting is restored. */
+acspgemm_status acspgemm_multiply_budget(acspgemm_plan plan, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
+                                         acspgemm_dtype dtype, void* stream, acspgemm_csr_out* C, int* npieces,
+                                         int* nrestarts);
+
 /* Galerkin triple product C = R·(A·P) as two ordered AC-SpGEMMs (SURVEY §8(f)-2,
  * reading R24: the association R·(A·P)).  A·P lives in temporary device memory that is
  * released before return; C is allocated like acspgemm_multiply (cudaMallocAsync on

@@ -63,6 +63,9 @@ SIGNATURES = {
                                          ctypes.c_int]),
     "acspgemm_multiply_host": (ctypes.c_int, [VP, ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.c_int, VP,
                                               ctypes.c_int, ctypes.POINTER(CsrOut), I64]),
+    "acspgemm_multiply_budget": (ctypes.c_int, [VP, ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.c_int, VP,
+                                                ctypes.POINTER(CsrOut), ctypes.POINTER(ctypes.c_int),
+                                                ctypes.POINTER(ctypes.c_int)]),
     "acspgemm_rap": (ctypes.c_int, [ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn), ctypes.POINTER(CsrIn),
                                     ctypes.POINTER(CsrOut), VP, ctypes.c_int]),
     "acspgemm_free_csr": (ctypes.c_int, [ctypes.POINTER(CsrOut), VP]),

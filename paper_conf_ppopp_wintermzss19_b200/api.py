@@ -180,6 +180,33 @@ class Plan:
                                                 _stream_ptr(stream)), "acspgemm_numeric_update")
         return C
 
+    def multiply_budget(self, A: DeviceCSR, B: DeviceCSR, stream=None):
+        """C = A·B within this plan's pool_limit_bytes through acspgemm_multiply_budget:
+        pieces of whole canonical segments, a piece over budget retried on fewer segments
+        (a "restart").  Bit-identical to multiply().  Returns ((row_ptr, col, val) as host
+        numpy arrays, pieces, restarts)."""
+        if A.dtype != B.dtype:
+            raise TypeError("A and B must have the same value dtype")
+        a, b = _csr_in(A), _csr_in(B)
+        c = CsrOut()
+        npc, nrs = ctypes.c_int(0), ctypes.c_int(0)
+        st = _stream_ptr(stream)
+        check(self._lib.acspgemm_multiply_budget(self._h, ctypes.byref(a), ctypes.byref(b), _dtype_code(A.dtype), st,
+                                                 ctypes.byref(c), ctypes.byref(npc), ctypes.byref(nrs)),
+              "acspgemm_multiply_budget")
+        try:
+            rp = np.empty(c.rows + 1, dtype=np.int32)
+            col = np.empty(c.nnz, dtype=np.int32)
+            val = np.empty(c.nnz, dtype=np.float64 if A.dtype == torch.float64 else np.float32)
+            torch.cuda.synchronize()
+            _memcpy_d2h(rp, c.row_ptr)
+            _memcpy_d2h(col, c.col_idx)
+            _memcpy_d2h(val, c.val)
+            return (rp, col, val), int(npc.value), int(nrs.value)
+        finally:
+            check(self._lib.acspgemm_free_csr(ctypes.byref(c), st), "acspgemm_free_csr")
+            torch.cuda.synchronize()
+
     def multiply_host(self, A, B, out=None, pieces: int = 4, stream=None):
         """End to end through acspgemm_multiply_host: A and B on the host (objects with
         rows, cols, row_ptr, col, val as numpy arrays or CPU tensors; int32 indices),

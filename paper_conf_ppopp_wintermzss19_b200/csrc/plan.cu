@@ -17,6 +17,7 @@
 #include <new>
 #include <string>
 #include <vector>
+#include <array>
 
 #include <algorithm>
 
@@ -103,6 +104,8 @@ struct acspgemm_plan_s {
   int rec_dtype = -1;
   cudaGraphExec_t gexec = nullptr;
   const void* gkey[9] = {};
+  // acspgemm_multiply_budget: the pieces' C buffers (row_ptr, col, val), kept for reuse
+  std::vector<std::array<DevBuf, 3>> bp;
 };
 
 namespace {
@@ -777,6 +780,7 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
                   &p->g_base, &p->g_tcol, &p->g_tval, &p->g_tcnt, &p->hdone, &p->esc_list,
                   &p->esc_list_small};
   for (DevBuf* b : bs) free_buf(*b);
+  for (auto& pb : p->bp) for (DevBuf& b : pb) free_buf(b);
   if (p->gexec) cudaGraphExecDestroy(p->gexec);
   for (int i = 0; i < 3; ++i) {
     free_buf(p->hp_a[i]);
@@ -930,6 +934,104 @@ acspgemm_status acspgemm_rap(const acspgemm_csr_in* R, const acspgemm_csr_in* A,
   acspgemm_free_csr(&AP, stream);
   if (s == ACSPGEMM_OK) ACS_CUDA(cudaStreamSynchronize(reinterpret_cast<cudaStream_t>(stream)));
   return s;
+}
+
+acspgemm_status acspgemm_multiply_budget(acspgemm_plan p, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
+                                         acspgemm_dtype dtype, void* stream, acspgemm_csr_out* C, int* npieces,
+                                         int* nrestarts) {
+  if (!p || !C) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
+  acspgemm_status s;
+  if ((s = check_in(A, "A")) != ACSPGEMM_OK) return s;
+  if ((s = check_in(B, "B")) != ACSPGEMM_OK) return s;
+  if (dtype != ACSPGEMM_F32 && dtype != ACSPGEMM_F64) return set_err(ACSPGEMM_ERR_INVALID_ARG, "bad dtype");
+  if (A->cols != B->rows) return set_err(ACSPGEMM_ERR_DIM_MISMATCH, "A.cols != B.rows");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const size_t vb = dtype == ACSPGEMM_F64 ? 8 : 4;
+  const int S = p->opt.num_segments;
+  int pieces = 0, restarts = 0;
+  C->rows = A->rows;
+  C->cols = B->cols;
+  C->nnz = 0;
+  C->row_ptr = nullptr; C->col_idx = nullptr; C->val = nullptr;
+  if (A->rows == 0 || A->nnz == 0 || B->nnz == 0) {         // no entries: one empty piece
+    int64_t nnz = 0;
+    if ((s = symbolic_impl(p, A, B, dtype, st, &nnz)) != ACSPGEMM_OK) return s;
+    ACS_CUDA(cudaMallocAsync((void**)&C->row_ptr, sizeof(int32_t) * (A->rows + 1), st));
+    if ((s = numeric_impl(p, C, st)) != ACSPGEMM_OK) return s;
+    if (npieces) *npieces = 1;
+    if (nrestarts) *nrestarts = 0;
+    ACS_CUDA(cudaStreamSynchronize(st));
+    return ACSPGEMM_OK;
+  }
+  HostPipeGuard guard(p, st);
+  // canonical segments of A: row and nonzero boundaries (one read-back)
+  int64_t seg[2 * (MAX_SEGMENTS + 1)];
+  {
+    ACS_ENSURE(p->seg, sizeof(int64_t) * (4 * (MAX_SEGMENTS + 1) + 2));
+    int64_t* sd = ptr<int64_t>(p->seg);
+    const CsrView Av{A->rows, A->cols, A->row_ptr, A->col_idx, A->val};
+    launch_segments(Av, S, nullptr, sd, reinterpret_cast<int32_t*>(sd + 4 * (MAX_SEGMENTS + 1)), st);
+    ACS_CUDA(cudaGetLastError());
+    ACS_CUDA(cudaMemcpyAsync(seg, sd, sizeof(int64_t) * 2 * (MAX_SEGMENTS + 1), cudaMemcpyDeviceToHost, st));
+    ACS_CUDA(cudaStreamSynchronize(st));
+  }
+  const int64_t* seg_nz = seg + (MAX_SEGMENTS + 1);
+  struct Piece { int64_t r0, rows, nnz; };
+  std::vector<Piece> out;
+  int64_t off = 0;
+  for (int s0 = 0; s0 < S;) {
+    int s1 = S;
+    int64_t nnz_g = 0;
+    for (;;) {                               // the largest run of whole segments within budget
+      const int64_t r0 = seg[s0], r1 = seg[s1];
+      p->nseg_explicit = s1 - s0;
+      for (int i = 0; i <= s1 - s0; ++i) p->seg_rows_explicit[i] = seg[s0 + i] - r0;
+      const acspgemm_csr_in V{r1 - r0, A->cols, seg_nz[s1] - seg_nz[s0], A->row_ptr + r0, A->col_idx, A->val};
+      s = symbolic_impl(p, &V, B, dtype, st, &nnz_g);
+      if (s == ACSPGEMM_OK) break;
+      if (s != ACSPGEMM_ERR_OUT_OF_MEMORY || s1 - s0 == 1) return s;
+      ++restarts;                            // pool over budget: retry on fewer segments
+      s1 = s0 + (s1 - s0) / 2;
+    }
+    if (off + nnz_g >= (int64_t(1) << 31)) return set_err(ACSPGEMM_ERR_INDEX_OVERFLOW, "nnz(C) >= 2^31");
+    Piece q{seg[s0], seg[s1] - seg[s0], nnz_g};
+    if (p->bp.size() <= out.size()) p->bp.emplace_back();
+    std::array<DevBuf, 3>& pb = p->bp[out.size()];
+    if ((s = ensure(pb[0], sizeof(int32_t) * (q.rows + 1))) != ACSPGEMM_OK ||
+        (s = ensure(pb[1], sizeof(int32_t) * nnz_g)) != ACSPGEMM_OK || (s = ensure(pb[2], vb * nnz_g)) != ACSPGEMM_OK)
+      return s;
+    acspgemm_csr_out Cg{q.rows, B->cols, nnz_g, ptr<int32_t>(pb[0]), ptr<int32_t>(pb[1]), pb[2].p};
+    out.push_back(q);
+    if ((s = numeric_impl(p, &Cg, st, (int32_t)off)) != ACSPGEMM_OK) return s;
+    off += nnz_g;
+    ++pieces;
+    s0 = s1;
+  }
+  // concatenate the pieces into C (allocated like acspgemm_multiply)
+  cudaError_t e = cudaMallocAsync((void**)&C->row_ptr, sizeof(int32_t) * (A->rows + 1), st);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&C->col_idx, sizeof(int32_t) * (off > 0 ? off : 1), st);
+  if (e == cudaSuccess) e = cudaMallocAsync(&C->val, vb * (off > 0 ? off : 1), st);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    acspgemm_free_csr(C, stream);
+    return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, std::string("cudaMallocAsync: ") + cudaGetErrorString(e));
+  }
+  int64_t o = 0;
+  for (size_t g = 0; g < out.size(); ++g) {
+    const Piece& q = out[g];
+    std::array<DevBuf, 3>& pb = p->bp[g];
+    ACS_CUDA(cudaMemcpyAsync(C->row_ptr + q.r0, pb[0].p, sizeof(int32_t) * (q.rows + 1), cudaMemcpyDeviceToDevice, st));
+    if (q.nnz > 0) {
+      ACS_CUDA(cudaMemcpyAsync(C->col_idx + o, pb[1].p, sizeof(int32_t) * q.nnz, cudaMemcpyDeviceToDevice, st));
+      ACS_CUDA(cudaMemcpyAsync(static_cast<char*>(C->val) + vb * o, pb[2].p, vb * q.nnz, cudaMemcpyDeviceToDevice, st));
+    }
+    o += q.nnz;
+  }
+  ACS_CUDA(cudaStreamSynchronize(st));
+  C->nnz = off;
+  if (npieces) *npieces = pieces;
+  if (nrestarts) *nrestarts = restarts;
+  return ACSPGEMM_OK;
 }
 
 acspgemm_status acspgemm_multiply_host(acspgemm_plan p, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
