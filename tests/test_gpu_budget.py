@@ -48,3 +48,19 @@ def test_budget_too_small(cuda_available):
     with pytest.raises(p.AcspgemmError) as e:
         plan.multiply_budget(dA, dA)
     assert e.value.status == 4                  # OUT_OF_MEMORY: one segment exceeds the budget
+
+
+def test_budget_empty_and_update_empty(cuda_available):
+    """Empty products through the budget and the update paths."""
+    from synth import CSR, random_csr
+    p = pkg()
+    A = CSR(5, 7, np.zeros(6, np.int32), np.zeros(0, np.int32), np.zeros(0))
+    B = random_csr(7, 4, 0.5, seed=1)
+    dA, dB = p.DeviceCSR.from_host(A, "cuda"), p.DeviceCSR.from_host(B, "cuda")
+    plan = p.Plan(pool_limit_bytes=1 << 20)
+    (rp, col, val), pieces, restarts = plan.multiply_budget(dA, dB)
+    assert (rp == 0).all() and len(col) == 0 and pieces == 1 and restarts == 0
+    C = plan.multiply(dA, dB)
+    plan.numeric_update(dA, dB, C)
+    torch.cuda.synchronize()
+    assert (C.row_ptr.cpu().numpy() == 0).all() and C.nnz == 0
