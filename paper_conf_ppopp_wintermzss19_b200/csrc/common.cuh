@@ -42,7 +42,10 @@ constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)
 constexpr int SEARCH_MAXP = 1024;            // Search Merge limit; longer chunk lists: dense slices (R30)
 constexpr int GIANT_SLICE = 4096;            // columns per dense-slice CTA
 constexpr int DENSE_SPAN_RATIO = 16;         // dense slices when span <= 16 x pre-merge elements
-constexpr int PAIR_MAX = 512;
+#ifndef ACS_PAIR_MAX
+#define ACS_PAIR_MAX 512
+#endif
+constexpr int PAIR_MAX = ACS_PAIR_MAX;     // two-chunk rows up to this many elements: one warp each (k_pair_merge)
 // hash accumulator (hash.cu, reading R31)
 #ifndef ACS_HASH_WARPS
 #define ACS_HASH_WARPS 4
