@@ -7,5 +7,4 @@ for l in sys.stdin:
     except: continue
     print(d['workload'], d['dtype'], round(d['ms_per_multiply'],2), {k: round(d['stages_ms'][k],2) for k in ('ESC','MM','PM','CC')})
 "
-  ACSPGEMM_LIB=$PWD/$lib python scratch/strat.py f64 128 esc 2>&1 | cut -c1-120
 done
