@@ -87,6 +87,7 @@ __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cac
     rp_cache[t] = r <= rowsA ? arp[r] : INT_MAX;
   }
   __syncthreads();
+  int prev = 0;                          // local row of this thread's previous entry
 #pragma unroll
   for (int j = 0; j < NPT; ++j) {
     const int e = tid * NPT + j;
@@ -95,11 +96,20 @@ __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cac
       const int nz = nzb + e;
       int r;
       if (nz < rp_cache[NPB]) {
-        int lo = 0, hi = NPB - 1;
-        while (lo < hi) {
-          const int mid = (lo + hi + 1) >> 1;
-          if (rp_cache[mid] <= nz) lo = mid; else hi = mid - 1;
+        // consecutive entries: a few steps on from the previous entry's row, else a
+        // binary search over the rest (rp_cache[lo] <= nz < rp_cache[lo + 1])
+        int lo = prev;
+#pragma unroll
+        for (int step = 0; step < 2; ++step)
+          if (rp_cache[lo + 1] <= nz) ++lo;
+        if (rp_cache[lo + 1] <= nz) {
+          int hi = NPB - 1;
+          while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (rp_cache[mid] <= nz) lo = mid; else hi = mid - 1;
+          }
         }
+        prev = lo;
         r = r0 + lo;
       } else {
         int64_t lo = (int64_t)r0 + NPB, hi = rowsA - 1;
