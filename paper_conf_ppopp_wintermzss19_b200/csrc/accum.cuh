@@ -48,7 +48,7 @@ __device__ __forceinline__ V block_exclusive_sum_nt(V x, V* scratch, V* total) {
 //   * the block's rows are numbered by rank: row_first[lr] = first compacted entry of
 //     local row lr (row_first[nrows] = nent), row_of[lr] = the row of A (and C).
 // rp_cache needs NPB + 1 ints and may alias other storage after the call; scratch needs
-// NT/32 + 1 ints.  Ends with a __syncthreads().  Returns whether this thread saw a B row
+// 2 (NT/32 + 1) ints, 8-byte aligned.  Ends with a __syncthreads().  Returns whether this thread saw a B row
 // longer than 32 entries.
 template <typename T, typename E, int NT = THREADS>
 __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cache, int* row_of, int* row_first,
@@ -135,9 +135,13 @@ __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cac
     psum += len[j];
     longb |= len[j] > 32;
   }
-  int tot_packed;
-  int ex = block_exclusive_sum_nt<NT, int>(packed, scratch, &tot_packed);   // barriers: reads above done
-  int pex = block_exclusive_sum_nt<NT, int>(psum, scratch, &total);
+  // one scan for both: (rows, entries) in the high word, products in the low word
+  long long tot2;
+  const long long ex2 = block_exclusive_sum_nt<NT, long long>(((long long)packed << 32) | (long long)psum,
+                                                              reinterpret_cast<long long*>(scratch), &tot2);
+  int ex = (int)(ex2 >> 32), pex = (int)(ex2 & 0xFFFFFFFFll);
+  const int tot_packed = (int)(tot2 >> 32);
+  total = (int)(tot2 & 0xFFFFFFFFll);
   nrows = tot_packed & 0xFFFF;
   nent = tot_packed >> 16;
 #pragma unroll

@@ -99,7 +99,7 @@ struct DictSmem {
   } u;
   int wrow[DICT_WARPS + 1];
   int wout[DICT_WARPS][5];
-  int scratch[40];
+  alignas(8) int scratch[40];
   int nd, cmin, cmax, bad;
 };
 static_assert(DICT_DMAX % 32 == 0, "the dummy slots lie outside the emitted windows");

@@ -51,7 +51,7 @@ struct RowsSmem {
   } u;
   int wrow[ROWS_WARPS + 1];
   int wout[ROWS_WARPS][5];
-  int scratch[40];
+  alignas(8) int scratch[40];
   int flag;
 };
 
