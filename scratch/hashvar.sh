@@ -1,4 +1,5 @@
 #!/bin/bash
-for lib in paper_conf_ppopp_wintermzss19_b200/libacspgemm_pw3.so paper_conf_ppopp_wintermzss19_b200/libacspgemm_pw4.so paper_conf_ppopp_wintermzss19_b200/libacspgemm_nopipe.so; do
+for lib in paper_conf_ppopp_wintermzss19_b200/libacspgemm*.so; do
   ACSPGEMM_LIB=$PWD/$lib python scratch/strat.py f64 128 hash 2>&1 | cut -c1-140
+  ACSPGEMM_LIB=$PWD/$lib python scratch/strat.py f32 128 hash 2>&1 | cut -c1-140
 done
