@@ -13,7 +13,9 @@
  *   several chunks -> row-pointer prefix sum -> chunk copy into C (§3.5).
  * Determinism: the block decomposition is fixed by A's nonzeros and the canonical
  *   segments; chunk slots are allocated per block (no atomics decide any placement or
- *   order); sums follow a fixed scan tree.  Results are bit-identical run to run and
+ *   order); every sum follows a fixed order (AC-ESC: the compaction scan tree of Alg. 3;
+ *   the adaptive accumulators: the left fold of a row's products in A-entry order).
+ *   Results are bit-identical run to run and
  *   for any split of the segments over GPUs ("bit-stable", L34, L198, L430).
  *
  * Conventions for every entry point:

@@ -30,8 +30,18 @@ def _stale(obj: str, deps) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
+def _flags_changed() -> bool:
+    """True when the nvcc flags differ from the ones the objects in BUILD were built with
+    (a -D knob in ACS_EXTRA_NVCC_FLAGS must not reuse objects of another variant)."""
+    stamp = os.path.join(BUILD, "FLAGS")
+    want = " ".join(FLAGS)
+    have = open(stamp).read() if os.path.exists(stamp) else None
+    return have != want
+
+
 def build(verbose: bool = False, ptxas_v: bool = False, force: bool = False) -> str:
     os.makedirs(BUILD, exist_ok=True)
+    force = force or _flags_changed()
     headers = [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith(".cuh")]
     headers.append(os.path.join(os.path.dirname(HERE), "include", "acspgemm.h"))
     jobs = []
@@ -50,6 +60,8 @@ def build(verbose: bool = False, ptxas_v: bool = False, force: bool = False) -> 
                 sys.stderr.write(r.stdout + r.stderr)
             if r.returncode:
                 raise RuntimeError("nvcc failed: " + " ".join(cmd))
+    with open(os.path.join(BUILD, "FLAGS"), "w") as f:
+        f.write(" ".join(FLAGS))
     objs = [os.path.join(BUILD, s.replace(".cu", ".o")) for s in SOURCES]
     if force or jobs or _stale(SO, objs):
         cmd = [NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", SO] + objs + ["-lcudart"]

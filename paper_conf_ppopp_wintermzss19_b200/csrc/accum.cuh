@@ -137,7 +137,8 @@ __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cac
   }
   // one scan for both: (rows, entries) in the high word, products in the low word
   long long tot2;
-  const long long ex2 = block_exclusive_sum_nt<NT, long long>(((long long)packed << 32) | (long long)psum,
+  // (a block's products are < 2^31: the symbolic pass refuses larger blocks, k_block_bounds)
+  const long long ex2 = block_exclusive_sum_nt<NT, long long>(((long long)packed << 32) | (long long)(uint32_t)psum,
                                                               reinterpret_cast<long long*>(scratch), &tot2);
   int ex = (int)(ex2 >> 32), pex = (int)(ex2 & 0xFFFFFFFFll);
   const int tot_packed = (int)(tot2 >> 32);

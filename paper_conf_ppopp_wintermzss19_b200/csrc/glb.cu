@@ -15,17 +15,16 @@ namespace acs {
 // seg layout: [0, MAX_SEGMENTS] rows | [MAX_SEGMENTS+1, ...] first nonzero | block base
 constexpr int SEG_STRIDE = MAX_SEGMENTS + 1;
 
-__global__ void k_segments(const int32_t* __restrict__ rp, int64_t rows, int nseg,
-                           const int64_t* __restrict__ explicit_rows, int64_t* __restrict__ seg,
-                           int32_t* __restrict__ nblocks) {
+__global__ void k_segments(const int32_t* __restrict__ rp, int64_t rows, int nseg, SegRows explicit_rows,
+                           int64_t* __restrict__ seg, int32_t* __restrict__ nblocks) {
   __shared__ int64_t s_rows[SEG_STRIDE], s_nz[SEG_STRIDE];
   const int s = threadIdx.x;
   const int64_t base = rp[0];
   const int64_t nnz = (int64_t)rp[rows] - base;
   if (s <= nseg) {
     int64_t r;
-    if (explicit_rows) {
-      r = explicit_rows[s];
+    if (explicit_rows.n > 0) {
+      r = explicit_rows.r[s];
     } else if (s == 0) {
       r = 0;
     } else if (s == nseg) {
@@ -56,7 +55,7 @@ __global__ void k_segments(const int32_t* __restrict__ rp, int64_t rows, int nse
   }
 }
 
-void launch_segments(const CsrView& A, int nseg, const int64_t* explicit_rows, int64_t* seg,
+void launch_segments(const CsrView& A, int nseg, const SegRows& explicit_rows, int64_t* seg,
                      int32_t* nblocks_dev, cudaStream_t st) {
   k_segments<<<1, 128, 0, st>>>(A.row_ptr, A.rows, nseg, explicit_rows, seg, nblocks_dev);
 }
@@ -112,7 +111,8 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
                                const int64_t* __restrict__ seg, const int32_t* __restrict__ nblocks_dev,
                                int64_t max_blocks, int32_t* __restrict__ nz_begin, int32_t* __restrict__ nz_end,
                                int64_t* __restrict__ products, int64_t* __restrict__ slots,
-                               int32_t* __restrict__ hash_ok, int64_t* __restrict__ ncand) {
+                               int32_t* __restrict__ hash_ok, int64_t* __restrict__ ncand,
+                               int64_t* __restrict__ max_products) {
   __shared__ int64_t s_nz[SEG_STRIDE], s_base[SEG_STRIDE];
   __shared__ int s_cand;
   for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
@@ -190,6 +190,9 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
       hok = mn > 0 && 4 * ov >= mn;
     }
     if (lane == 0) {
+      // the block kernels count a block's products in 32 bits (fetch_block): a block of
+      // >= 2^31 products is refused by the symbolic pass (read back with the totals)
+      if (sum > (int64_t)INT_MAX) atomicMax(reinterpret_cast<unsigned long long*>(max_products), (unsigned long long)sum);
       if (hash_ok) hash_ok[b] = hok;
       if (hok) atomicAdd(&s_cand, 1);
       products[b] = sum;
@@ -206,12 +209,13 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
 
 void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* nzb, int32_t* nze,
-                         int64_t* products, int64_t* slots, int32_t* hash_ok, int64_t* ncand, cudaStream_t st) {
+                         int64_t* products, int64_t* slots, int32_t* hash_ok, int64_t* ncand,
+                         int64_t* max_products, cudaStream_t st) {
   if (max_blocks == 0) return;
   const int T = 256, WPB = T / 32;
   k_block_bounds<<<(unsigned)((max_blocks + WPB - 1) / WPB), T, 0, st>>>(
       A.row_ptr, A.col, B.row_ptr, B.col, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots, hash_ok,
-      ncand);
+      ncand, max_products);
 }
 
 // Canonical-CSR check (reading R3): row_ptr monotone, columns strictly increasing and

@@ -14,9 +14,14 @@ struct CsrView {              // device CSR view; row_ptr values index col/val d
 };
 
 // ---- stage 1: global load balancing (glb.cu) ----------------------------------
-// seg_rows_host: explicit segment row boundaries (nseg+1) or nullptr for canonical.
+// Explicit segment row boundaries, passed BY VALUE as a kernel argument (so a captured
+// graph and an asynchronous launch keep their own copy); n == 0: canonical segments.
+struct SegRows {
+  int32_t n;
+  int64_t r[MAX_SEGMENTS + 1];
+};
 // Writes seg tables to `seg` (device, int64[4*(MAX_SEGMENTS+1)]): rows | nz | block base.
-void launch_segments(const CsrView& A, int nseg, const int64_t* seg_rows_dev_or_null,
+void launch_segments(const CsrView& A, int nseg, const SegRows& explicit_rows,
                      int64_t* seg, int32_t* nblocks_dev, cudaStream_t st);
 void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* block_row_starts,
                 int64_t max_blocks, cudaStream_t st);
@@ -24,7 +29,9 @@ void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* blk_nz_begin,
                          int32_t* blk_nz_end, int64_t* blk_products, int64_t* blk_slots,
                          int32_t* blk_hash_ok /* nullable: hash-accumulator candidates (R31) */,
-                         int64_t* ncand /* nullable: their count (zeroed by the caller) */, cudaStream_t st);
+                         int64_t* ncand /* nullable: their count (zeroed by the caller) */,
+                         int64_t* max_products /* atomicMax of block products > INT_MAX (zeroed) */,
+                         cudaStream_t st);
 
 // ---- device-wide exclusive scan (scan.cu) --------------------------------------
 // out[i] = sum_{j<i} in[j] for i < n, total -> *total_dev.  tmp needs scan_tmp_elems(n).

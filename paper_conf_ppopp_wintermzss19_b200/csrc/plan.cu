@@ -57,8 +57,8 @@ struct DevBuf {
   size_t bytes = 0;
 };
 
-// mapped host buffer h_scal: [0, 32) read-backs, [32, 97) explicit segment rows (read by
-// the segments kernel), [97, 162) segment boundaries read back for acspgemm_info
+// mapped host buffer h_scal: [0, 32) read-backs, [32, 97) unused, [97, 162) segment
+// boundaries read back for acspgemm_info
 constexpr int H_SEG_ROWS = 32;
 constexpr int H_SEG_INFO = H_SEG_ROWS + MAX_SEGMENTS + 1;
 constexpr int H_SCAL_WORDS = H_SEG_INFO + MAX_SEGMENTS + 1;
@@ -73,7 +73,7 @@ struct acspgemm_plan_s {
   int nseg_explicit = 0;
   int64_t seg_rows_explicit[MAX_SEGMENTS + 1];
   // buffers
-  DevBuf seg, seg_rows, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base;
+  DevBuf seg, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base;
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan, hdone, esc_list, esc_list_small;
@@ -163,7 +163,7 @@ acspgemm_status check_in(const acspgemm_csr_in* M, const char* name) {
 }
 
 int64_t helper_bytes(acspgemm_plan p) {
-  DevBuf* bs[] = {&p->seg, &p->seg_rows, &p->scal, &p->brs, &p->nzb, &p->nze, &p->bprod, &p->bslot,
+  DevBuf* bs[] = {&p->seg, &p->scal, &p->brs, &p->nzb, &p->nze, &p->bprod, &p->bslot,
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->descs, &p->dense, &p->sflag,
                   &p->spos, &p->shared, &p->row_count, &p->row_ptr, &p->scan_tmp, &p->kflag, &p->kpos,
                   &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
@@ -256,16 +256,15 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   if (nseg > MAX_SEGMENTS) nseg = MAX_SEGMENTS;
   const int64_t max_blocks = (A->nnz + NPB - 1) / NPB + nseg;
   ACS_ENSURE(p->seg, sizeof(int64_t) * 3 * (MAX_SEGMENTS + 1));
-  ACS_ENSURE(p->seg_rows, sizeof(int64_t) * (MAX_SEGMENTS + 1));
-  const int64_t* explicit_rows = nullptr;
+  SegRows explicit_rows;
+  explicit_rows.n = 0;
   if (p->nseg_explicit > 0) {
     if (p->seg_rows_explicit[p->nseg_explicit] != A->rows)
       return set_err(ACSPGEMM_ERR_INVALID_ARG, "explicit segments do not end at A.rows");
-    // through mapped host memory (no copy engine: see launch_read_back); the previous
-    // symbolic has synchronised, so no kernel still reads the old values
-    int64_t* hs = p->h_scal + H_SEG_ROWS;
-    for (int i = 0; i <= nseg; ++i) hs[i] = p->seg_rows_explicit[i];
-    explicit_rows = hs;
+    // by value in the kernel arguments: a captured graph (numeric_update) keeps this
+    // copy, whatever later calls do to the plan's segments
+    explicit_rows.n = nseg + 1;
+    for (int i = 0; i <= nseg; ++i) explicit_rows.r[i] = p->seg_rows_explicit[i];
   }
   ACS_ENSURE(p->brs, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->nzb, sizeof(int32_t) * max_blocks);
@@ -288,10 +287,10 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   tl_launches += 1;
   launch_glb(Av, nseg, ptr<int64_t>(p->seg), ptr<int32_t>(p->brs), max_blocks, st);
   tl_launches += 1;
-  ACS_CUDA(cudaMemsetAsync(scal + 3, 0, sizeof(int64_t), st));   // hash candidates (R31)
+  ACS_CUDA(cudaMemsetAsync(scal + 3, 0, 2 * sizeof(int64_t), st));   // hash candidates (R31), max block products
   launch_block_bounds(Av, Bv, nseg, ptr<int64_t>(p->seg), nblocks_dev, max_blocks, ptr<int32_t>(p->nzb),
                       ptr<int32_t>(p->nze), ptr<int64_t>(p->bprod), ptr<int64_t>(p->bslot),
-                      p->opt.strategy != ACSPGEMM_STRATEGY_ESC ? ptr<int32_t>(p->hdone) : nullptr, scal + 3, st);
+                      p->opt.strategy != ACSPGEMM_STRATEGY_ESC ? ptr<int32_t>(p->hdone) : nullptr, scal + 3, scal + 4, st);
   tl_launches += 1;
   launch_scan_i64(ptr<int64_t>(p->bprod), ptr<int64_t>(p->pool_off), max_blocks, scal + 0, ptr<int64_t>(p->scan_tmp), st);
   launch_scan_i64(ptr<int64_t>(p->bslot), ptr<int64_t>(p->desc_off), max_blocks, scal + 1, ptr<int64_t>(p->scan_tmp), st);
@@ -304,8 +303,11 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     launch_read_back(p->seg.p, p->h_scal + H_SEG_INFO, (int)sizeof(int64_t) * (nseg + 1), st);
     tl_launches += 1;
   }
-  if ((s = sync_read(p, scal, 4, st)) != ACSPGEMM_OK) return s;
+  if ((s = sync_read(p, scal, 5, st)) != ACSPGEMM_OK) return s;
   const int64_t products = p->h_scal[0], slots = p->h_scal[1], nblocks = p->h_scal[2], ncand = p->h_scal[3];
+  if (p->h_scal[4] > 0)
+    return set_err(ACSPGEMM_ERR_INDEX_OVERFLOW, "a block of NPB nonzeros of A has " + std::to_string(p->h_scal[4]) +
+                                                    " >= 2^31 products (32-bit block counters)");
   p->info.products = products;
   p->info.nblocks = nblocks;
   p->info.nsegments = nseg;
@@ -771,7 +773,7 @@ acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options
 void acspgemm_plan_destroy(acspgemm_plan p) {
   if (!p) return;
   cudaDeviceSynchronize();
-  DevBuf* bs[] = {&p->seg, &p->seg_rows, &p->scal, &p->brs, &p->nzb, &p->nze, &p->bprod, &p->bslot,
+  DevBuf* bs[] = {&p->seg, &p->scal, &p->brs, &p->nzb, &p->nze, &p->bprod, &p->bslot,
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->pool_col, &p->pool_val,
                   &p->descs, &p->dense, &p->sflag, &p->spos, &p->shared, &p->row_count, &p->row_ptr,
                   &p->scan_tmp, &p->kflag, &p->kpos, &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan,
@@ -821,7 +823,7 @@ acspgemm_status acspgemm_canonical_segments(const acspgemm_csr_in* A, int nseg, 
   Scratch<int64_t> seg;
   ACS_CUDA(cudaMalloc(&seg.d, sizeof(int64_t) * (3 * (MAX_SEGMENTS + 1) + 2)));
   const CsrView Av{A->rows, A->cols, A->row_ptr, A->col_idx, A->val};
-  launch_segments(Av, nseg, nullptr, seg.d, reinterpret_cast<int32_t*>(seg.d + 3 * (MAX_SEGMENTS + 1)), st);
+  launch_segments(Av, nseg, SegRows{}, seg.d, reinterpret_cast<int32_t*>(seg.d + 3 * (MAX_SEGMENTS + 1)), st);
   ACS_CUDA(cudaGetLastError());
   ACS_CUDA(cudaMemcpyAsync(rows_host, seg.d, sizeof(int64_t) * (nseg + 1), cudaMemcpyDeviceToHost, st));
   ACS_CUDA(cudaStreamSynchronize(st));
@@ -970,7 +972,7 @@ acspgemm_status acspgemm_multiply_budget(acspgemm_plan p, const acspgemm_csr_in*
     ACS_ENSURE(p->seg, sizeof(int64_t) * (4 * (MAX_SEGMENTS + 1) + 2));
     int64_t* sd = ptr<int64_t>(p->seg);
     const CsrView Av{A->rows, A->cols, A->row_ptr, A->col_idx, A->val};
-    launch_segments(Av, S, nullptr, sd, reinterpret_cast<int32_t*>(sd + 4 * (MAX_SEGMENTS + 1)), st);
+    launch_segments(Av, S, SegRows{}, sd, reinterpret_cast<int32_t*>(sd + 4 * (MAX_SEGMENTS + 1)), st);
     ACS_CUDA(cudaGetLastError());
     ACS_CUDA(cudaMemcpyAsync(seg, sd, sizeof(int64_t) * 2 * (MAX_SEGMENTS + 1), cudaMemcpyDeviceToHost, st));
     ACS_CUDA(cudaStreamSynchronize(st));
@@ -1090,7 +1092,7 @@ acspgemm_status acspgemm_multiply_host(acspgemm_plan p, const acspgemm_csr_in* A
     ACS_ENSURE(p->seg, sizeof(int64_t) * (4 * (MAX_SEGMENTS + 1) + 2));
     int64_t* sd = ptr<int64_t>(p->seg);
     const CsrView Av{D[0].rows, D[0].cols, D[0].row_ptr, D[0].col_idx, D[0].val};
-    launch_segments(Av, S, nullptr, sd, reinterpret_cast<int32_t*>(sd + 4 * (MAX_SEGMENTS + 1)), st);
+    launch_segments(Av, S, SegRows{}, sd, reinterpret_cast<int32_t*>(sd + 4 * (MAX_SEGMENTS + 1)), st);
     tl_launches += 1;
     ACS_CUDA(cudaGetLastError());
     ACS_CUDA(cudaMemcpyAsync(seg, sd, sizeof(int64_t) * (S + 1), cudaMemcpyDeviceToHost, st));

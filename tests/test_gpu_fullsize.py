@@ -101,15 +101,37 @@ def test_cfg2_27pt_128_full(dt, cuda_available):
     check_rows(A, A, sample_rows(A, rp, 1500, 1), (rp, col, val), 0, exact=True)
 
 
-def test_cfg3_rmat_full(cuda_available):
-    """configs[2]: R-MAT scale 20 (long skewed rows: Multi and Path Merge at scale).
-    nnz(C) = 581,442,205 (scipy); sampled rows incl. the 200 longest."""
-    A, _ = config("cfg3", np.float64)
-    (rp, col, val), info = gpu_full(A, A, np.float64)
+TOL = {np.float64: 1e-12, np.float32: 1e-5}
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_cfg3_rmat_full(dt, cuda_available):
+    """configs[2]: R-MAT scale 20 (long skewed rows: Multi and Path Merge at scale), in
+    fp64 and fp32 (L554: every matrix in float and double).  nnz(C) = 581,442,205
+    (scipy); sampled rows incl. the 200 longest and the segment
+    boundaries vs the oracle (on the dtype-rounded inputs)."""
+    A, _ = config("cfg3", dt)
+    (rp, col, val), info = gpu_full(A, A, dt)
     rowptr_invariants(rp, A.rows, 581442205)
     assert info["products"] == 585358301
     assert info["npath"] + info["nsearch"] > 0
-    check_rows(A, A, sample_rows(A, rp, 1500, 3), (rp, col, val), 1e-12, exact=False)
+    check_rows(A, A, sample_rows(A, rp, 1500, 3), (rp, col, val), TOL[dt], exact=False)
+
+
+def test_graph500_rmat_s18_full(cuda_available):
+    """§8(f)-1 stress: Graph500-parameter R-MAT (a, b, c = .57, .19, .19; SURVEY §8(c)
+    reading 23) at scale 18, ef 16 -- max out-degree ~15.8k, ~2.9 G products, rows of
+    C spread over hundreds of chunks (Path / Search Merge, dense slices).  Structure
+    bit-exact and values within 1e-12 on sampled rows (the 200 longest included)."""
+    from synth import rmat
+    A = rmat(scale=18, edge_factor=16, abc=(0.57, 0.19, 0.19), values="uniform")
+    deg = np.diff(A.row_ptr.astype(np.int64))
+    assert deg.max() > 10000
+    (rp, col, val), info = gpu_full(A, A, np.float64)
+    rowptr_invariants(rp, A.rows)
+    assert info["products"] == oracle.products(A, A)
+    assert info["npath"] + info["nsearch"] > 0
+    check_rows(A, A, sample_rows(A, rp, 400, 18), (rp, col, val), 1e-12, exact=False)
 
 
 def test_cfg4_galerkin_rap_full(cuda_available):
@@ -131,11 +153,12 @@ def test_cfg4_galerkin_rap_full(cuda_available):
     assert (rp2 == A4.row_ptr).all() and (col2 == A4.col).all() and (val2 == 4 * A4.val).all()
 
 
-def test_cfg5_lp_full(cuda_available):
-    """configs[4]: LP-like 2²⁰ × 2²², 20 nnz/col, C = A·Aᵀ (Aᵀ precomputed).  Products =
-    2²²·20² exactly; sampled rows vs the oracle (fp64 tolerance)."""
-    A, At = config("cfg5", np.float64)
-    (rp, col, val), info = gpu_full(A, At, np.float64)
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_cfg5_lp_full(dt, cuda_available):
+    """configs[4]: LP-like 2²⁰ × 2²², 20 nnz/col, C = A·Aᵀ (Aᵀ precomputed), fp64 and
+    fp32.  Products = 2²²·20² exactly; sampled rows vs the oracle."""
+    A, At = config("cfg5", dt)
+    (rp, col, val), info = gpu_full(A, At, dt)
     rowptr_invariants(rp, A.rows)
     assert info["products"] == (1 << 22) * 400
-    check_rows(A, At, sample_rows(A, rp, 300, 5), (rp, col, val), 1e-12, exact=False)
+    check_rows(A, At, sample_rows(A, rp, 300, 5), (rp, col, val), TOL[dt], exact=False)

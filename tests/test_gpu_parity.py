@@ -370,8 +370,9 @@ def test_sort_compact_vs_alg3(seed, cuda_available):
     assert (oval[runend] == np.array([r[2] for r in ref])[runend]).all()
 
 
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
 @pytest.mark.parametrize("ncols_log2", [16, 24])
-def test_wide_column_ranges(ncols_log2, cuda_available):
+def test_wide_column_ranges(ncols_log2, dt, cuda_available):
     """Column ranges that need 32-bit sort words (16) and the split 32-bit + side-array
     words (24) in AC-ESC; B has few rows with columns spread over 2^ncols_log2.  (The
     oracle's dense accumulator is as wide as C: one oracle thread keeps it small.)"""
@@ -385,10 +386,10 @@ def test_wide_column_ranges(ncols_log2, cuda_available):
         cols.append(c)
     rows, cols = np.concatenate(rows), np.concatenate(cols)
     B = from_coo(K, ncols, rows, cols, rng.uniform(-1, 1, rows.size))
-    assert_parity(A, B, np.float64, oracle_threads=1)
+    assert_parity(A, B, dt, oracle_threads=1)
     Bi = from_coo(K, ncols, rows, cols, rng.integers(-3, 4, rows.size).astype(np.float64))
     Ai = random_rowlen_csr(600, K, rng.integers(1, 40, 600), seed=ncols_log2 + 1, values="int")
-    assert_parity(Ai, Bi, np.float64, exact=True, oracle_threads=1)
+    assert_parity(Ai, Bi, dt, exact=True, oracle_threads=1)
 
 
 def test_64bit_sort_words(cuda_available):
