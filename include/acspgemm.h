@@ -94,11 +94,11 @@ typedef struct {
   int collect_stage_times;   /* 1: record CUDA events between stages (acspgemm_stage_times) */
   int num_segments;          /* canonical segments S (default 8, max 64) */
   int strategy;              /* ACSPGEMM_STRATEGY_ADAPTIVE (default): each candidate block is tried
-                                by the column-dictionary accumulator (reading R33; fp32 only),
-                                then the hash accumulator (R31), and falls back to AC-ESC;
+                                by the hash accumulator (R31) and falls back to AC-ESC; blocks of
+                                short rows go to the per-row accumulator (R34);
                                 ACSPGEMM_STRATEGY_ESC: every block through AC-ESC;
                                 ACSPGEMM_STRATEGY_HASH: hash accumulator, then AC-ESC;
-                                ACSPGEMM_STRATEGY_DICT: dictionary (any dtype), hash, AC-ESC.
+                                ACSPGEMM_STRATEGY_DICT: block dictionary (R33), hash, AC-ESC.
                                 ADAPTIVE, HASH and DICT give the same results bit for bit. */
 } acspgemm_options;
 

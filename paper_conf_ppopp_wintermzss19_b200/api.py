@@ -91,10 +91,10 @@ class Plan:
 
     def __init__(self, pool_limit_bytes: int = 0, validate: bool = False, stage_times: bool = False,
                  num_segments: int = 8, strategy: str = "adaptive"):
-        """strategy: "adaptive" (column-dictionary accumulator for fp32, then the hash
-        accumulator per candidate block, AC-ESC fallback; readings R33, R31), "hash" (no
-        dictionary), "dict" (dictionary for every dtype) -- these three give the same bits --
-        or "esc" (every block through AC-ESC)."""
+        """strategy: "adaptive" (hash accumulator per candidate block, per-row accumulator
+        for blocks of short rows, AC-ESC fallback; readings R31, R34), "hash" (the same path;
+        kept for the round-1 API), "dict" (column dictionary first, reading R33) -- these three give the
+        same bits -- or "esc" (every block through AC-ESC)."""
         if strategy not in _STRATEGIES:
             raise ValueError("strategy must be one of " + ", ".join(_STRATEGIES))
         lib = load()

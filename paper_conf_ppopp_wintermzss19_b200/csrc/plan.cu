@@ -366,8 +366,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   // column dictionary first (reading R33): by default for fp32 only -- with fp64 values its
   // per-warp accumulators allow 2 CTAs (16 warps) per SM and it measured slower than the
   // hash table (cfg2: 10.5 vs 10.1 ms; fp32: 7.8 vs 9.5 ms); both give the same bits
-  const bool use_dict = p->opt.strategy == ACSPGEMM_STRATEGY_DICT ||
-                        (p->opt.strategy == ACSPGEMM_STRATEGY_ADAPTIVE && !p->f64);
+  const bool use_dict = p->opt.strategy == ACSPGEMM_STRATEGY_DICT;
   if (ea.hash_done && ncand > 0 && use_dict) {
     launch_dict(ea, p->f64, st);
     tl_launches += nblocks > 0 ? 1 : 0;

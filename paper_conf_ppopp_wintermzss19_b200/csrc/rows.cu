@@ -82,7 +82,9 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
   T(*lv)[THREADS] = S.u.l.val;
   int out = 0, first_row = -1, last_row = -1, first_count = 0, last_count = 0;
   for (int r0 = rlo; r0 < rhi; r0 += 32) {
-    if (atomicOr(&S.flag, 0)) break;   // another warp abandoned the block (atomic: no race)
+    // another warp abandoned the block: one lane reads the flag, the warp follows it
+    // (per-lane atomics could disagree and split the warp)
+    if (__shfl_sync(0xffffffffu, lane == 0 ? atomicOr(&S.flag, 0) : 0, 0)) break;
     const int r = r0 + lane;
     int cnt = 0;
     bool over = false;

@@ -10,8 +10,8 @@ What pins it:
   * the fallbacks (dictionary wider than 768 columns, column span beyond 131,072, more
     than 7,168 staged B entries) leave the block to the hash accumulator with the same
     bits; structural zeros from cancellation are kept (reading R2);
-  * the default strategy uses the dictionary for fp32 and the hash table for fp64
-    (same bits); these tests force it with strategy "dict".
+  * the default strategy offers the blocks to the hash accumulator (same bits); these
+    tests force the dictionary with strategy "dict".
 """
 import numpy as np
 import pytest
@@ -89,7 +89,7 @@ def test_dict_stencil_all_blocks(dt, cuda_available):
     assert info_h["ndict_blocks"] == 0 and info_h["nhash_blocks"] == info["nblocks"]
     assert same_bytes(out, hsh)
     dflt, info_a = run(A, A, dt, strategy="adaptive")
-    assert info_a["ndict_blocks"] == (info["nblocks"] if dt == np.float32 else 0)
+    assert info_a["ndict_blocks"] == 0 and info_a["nhash_blocks"] == info["nblocks"]   # adaptive: hash (R31)
     assert same_bytes(out, dflt)
 
 
