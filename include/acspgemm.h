@@ -238,6 +238,20 @@ acspgemm_status acspgemm_stage_times(acspgemm_plan plan, float* ms_out, int n);
 /* Counters of the last multiply. */
 acspgemm_status acspgemm_plan_info(acspgemm_plan plan, acspgemm_info* info);
 
+/* Multiprocessor load (Table 3's "lowest multiprocessor load", mpL, L746-L760, L832).
+ * acspgemm_set_trace(plan, 1) makes the following symbolic passes record, for every block
+ * a stage-2 kernel processes, the SM it ran on (%smid) and its start / end time
+ * (%globaltimer); 0 turns it off (the default; recording costs two timer reads and three
+ * stores per block).  acspgemm_sm_load then reports, for kernel 0 = hash accumulator
+ * (k_hash), 1 = per-row accumulator (k_rows), 2 = AC-ESC (k_esc), 3 = small-tile AC-ESC:
+ * per SM the summed block time in ms (per_sm_ms, host, nsm entries; nullable) and
+ * *mpl = min over SMs / max over SMs of that busy time (1 = perfectly balanced; reading
+ * R36), and *nblocks_traced (nullable) = blocks the kernel processed.  Synchronous (reads
+ * the records back).  NOT_READY if the last symbolic was not traced. */
+acspgemm_status acspgemm_set_trace(acspgemm_plan plan, int enable);
+acspgemm_status acspgemm_sm_load(acspgemm_plan plan, int kernel, double* per_sm_ms, int nsm, double* mpl,
+                                 int64_t* nblocks_traced);
+
 /* Copy the last blockRowStarts array (Alg. 1 output, one int32 per block) to host. */
 acspgemm_status acspgemm_block_row_starts(acspgemm_plan plan, int32_t* host_out, int64_t n);
 

@@ -72,6 +72,9 @@ SIGNATURES = {
     "acspgemm_stage_times": (ctypes.c_int, [VP, ctypes.POINTER(ctypes.c_float), ctypes.c_int]),
     "acspgemm_plan_info": (ctypes.c_int, [VP, ctypes.POINTER(Info)]),
     "acspgemm_block_row_starts": (ctypes.c_int, [VP, PI32, I64]),
+    "acspgemm_set_trace": (ctypes.c_int, [VP, ctypes.c_int]),
+    "acspgemm_sm_load": (ctypes.c_int, [VP, ctypes.c_int, ctypes.POINTER(ctypes.c_double), ctypes.c_int,
+                                        ctypes.POINTER(ctypes.c_double), PI64]),
     "acspgemm_pool_estimate_bytes": (ctypes.c_double, [I64, I64, I64, I64, I64, ctypes.c_int]),
     "acspgemm_debug_work_distribution": (ctypes.c_int, [PI32, ctypes.c_int, PI32, ctypes.c_int, PI32, PI32, PI32]),
     "acspgemm_debug_sort_compact": (ctypes.c_int, [PI32, PI32, ctypes.POINTER(ctypes.c_double), ctypes.c_int,

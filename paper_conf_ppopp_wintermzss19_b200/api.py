@@ -251,6 +251,21 @@ class Plan:
         d["segment_rows"] = [inf.segment_rows[i] for i in range(inf.nsegments + 1)] if inf.nsegments else []
         return d
 
+    def set_trace(self, enable: bool = True) -> None:
+        """Record (SM, start, end) per block of the stage-2 kernels in the next multiplies."""
+        check(self._lib.acspgemm_set_trace(self._h, int(bool(enable))), "acspgemm_set_trace")
+
+    def sm_load(self, kernel: str = "hash") -> dict:
+        """Multiprocessor load of one kernel of the last traced multiply (Table 3's mpL):
+        {"mpl": min/max of the per-SM busy time, "per_sm_ms": [...], "blocks": n}."""
+        k = {"hash": 0, "rows": 1, "esc": 2, "esc_small": 3}[kernel]
+        nsm = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+        per = (ctypes.c_double * nsm)()
+        mpl = ctypes.c_double()
+        nb = ctypes.c_int64()
+        check(self._lib.acspgemm_sm_load(self._h, k, per, nsm, ctypes.byref(mpl), ctypes.byref(nb)), "acspgemm_sm_load")
+        return {"mpl": float(mpl.value), "per_sm_ms": [float(per[i]) for i in range(nsm)], "blocks": int(nb.value)}
+
     def stage_times(self) -> dict:
         buf = (ctypes.c_float * len(STAGES))()
         check(self._lib.acspgemm_stage_times(self._h, buf, len(STAGES)), "acspgemm_stage_times")

@@ -96,6 +96,26 @@ struct SharedRow {
 
 // ---------------------------------------------------------------- helpers --
 
+// Per-block trace for the multiprocessor-load report (Table 3's mpL, L760; acspgemm_sm_load):
+// tr[3b] = SM id, tr[3b+1] = start, tr[3b+2] = end (%globaltimer, ns).
+__device__ __forceinline__ uint64_t global_timer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ uint32_t sm_id() {
+  uint32_t s;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(s));
+  return s;
+}
+__device__ __forceinline__ void trace_block(uint64_t* tr, int64_t b, uint64_t t0) {
+  if (tr) {
+    tr[3 * b] = sm_id();
+    tr[3 * b + 1] = t0;
+    tr[3 * b + 2] = global_timer();
+  }
+}
+
 __device__ __forceinline__ int bit_width_u64(uint64_t x) { return x ? 64 - __clzll((long long)x) : 0; }
 
 template <typename T> struct ValueTraits;

@@ -399,7 +399,9 @@ __global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   EscSmem<T>& S = *reinterpret_cast<EscSmem<T>*>(smem_raw);
   if (!a.hash_done) {
+    const uint64_t t0 = a.trace ? global_timer() : 0;
     esc_block<T>(S, a, blockIdx.x);
+    if (threadIdx.x == 0) trace_block(a.trace, blockIdx.x, t0);
     return;
   }
   const int64_t n = *a.esc_count;
@@ -410,7 +412,9 @@ __global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
     const int i = S.s.misc[15];
     __syncthreads();
     if (i >= n) break;
+    const uint64_t t0 = a.trace ? global_timer() : 0;
     esc_block<T>(S, a, a.esc_list[i]);
+    if (threadIdx.x == 0) trace_block(a.trace, a.esc_list[i], t0);
     __syncthreads();                                  // shared memory is reused by the next block
   }
 }

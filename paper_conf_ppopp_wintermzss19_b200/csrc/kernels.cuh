@@ -66,6 +66,7 @@ struct EscArgs {
   int64_t* esc_count;           // adaptive: their number (zeroed before launch_hash)
   int64_t* esc_next;            // adaptive: grab counter of the persistent k_esc (zeroed)
   const int64_t* blk_products;  // per block product count
+  uint64_t* trace;              // nullable: per-block (SM, start, end) of this launch's kernel (mpL)
   int32_t* esc_list_small;      // adaptive: left blocks of <= CAP_SMALL products [nblocks]
   int64_t* esc_count_small;     // (zeroed) -- the small-tile AC-ESC's list, counter
   int64_t* esc_next_small;      // (zeroed)

@@ -78,6 +78,9 @@ struct acspgemm_plan_s {
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan, hdone, esc_list, esc_list_small;
   DevBuf lgiant, g_lo, g_nsl, g_base, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30): lists, spans, slices
+  DevBuf trace;                  // acspgemm_set_trace: per block (SM, start, end) x 4 kernels (mpL)
+  bool trace_on = false;
+  int64_t trace_blocks = 0;
   // acspgemm_multiply_host: device copies of A and B, two C piece buffers, copy stream
   DevBuf hp_a[3], hp_b[3], hp_c[2][3];
   cudaStream_t hp_cs = nullptr;
@@ -354,6 +357,15 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_CUDA(cudaMemsetAsync(scal + 28, 0, 2 * sizeof(int64_t), st));
   ea.blk_products = ptr<int64_t>(p->bprod);
   ea.esc_list_small = nullptr;
+  ea.trace = nullptr;
+  uint64_t* trace_base = nullptr;        // kernel k's records at trace_base + k * 3 * nblocks
+  if (p->trace_on && !p->replay) {
+    ACS_ENSURE(p->trace, sizeof(uint64_t) * 3 * 4 * nblocks);
+    ACS_CUDA(cudaMemsetAsync(p->trace.p, 0, sizeof(uint64_t) * 3 * 4 * nblocks, st));
+    trace_base = ptr<uint64_t>(p->trace);
+    p->trace_blocks = nblocks;
+  }
+  auto trace_of = [&](int k) { return trace_base ? trace_base + (int64_t)k * 3 * nblocks : nullptr; };
   ea.esc_count_small = scal + 30;
   ea.esc_next_small = scal + 31;
   if (p->opt.strategy != ACSPGEMM_STRATEGY_ESC) {
@@ -373,21 +385,26 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   }
   record(p, S_DICTEND, st);
   if (ea.hash_done && ncand > 0) {
+    ea.trace = trace_of(0);
     launch_hash(ea, p->f64, st);         // blocks k_dict left (reading R31)
     tl_launches += nblocks > 0 ? 1 : 0;
   }
   record(p, S_HASHEND, st);
   if (ea.hash_done) {
+    ea.trace = trace_of(1);
     launch_rows(ea, p->f64, st);         // blocks of short rows (reading R34)
     tl_launches += nblocks > 0 ? 1 : 0;
   }
   if (ea.hash_done) {
     launch_esc_lists(ea, st);
+    ea.trace = trace_of(3);
     acs_launch_esc_small(&ea, p->f64, st);
     tl_launches += nblocks > 0 ? 2 : 0;
   }
+  ea.trace = trace_of(2);
   launch_esc(ea, p->f64, st);
   tl_launches += nblocks > 0 ? 1 : 0;
+  ea.trace = nullptr;
   ACS_CUDA(cudaGetLastError());
 
   // ------------------------------------------------------------ MCC -----------
@@ -779,7 +796,7 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
                   &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
                   &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->lgiant, &p->g_lo, &p->g_nsl,
                   &p->g_base, &p->g_tcol, &p->g_tval, &p->g_tcnt, &p->hdone, &p->esc_list,
-                  &p->esc_list_small};
+                  &p->esc_list_small, &p->trace};
   for (DevBuf* b : bs) free_buf(*b);
   for (auto& pb : p->bp) for (DevBuf& b : pb) free_buf(b);
   if (p->gexec) cudaGraphExecDestroy(p->gexec);
@@ -1173,6 +1190,45 @@ acspgemm_status acspgemm_stage_times(acspgemm_plan p, float* ms_out, int n) {
     if (cudaEventElapsedTime(&ms, p->ev[a], p->ev[b]) != cudaSuccess) { cudaGetLastError(); ms = -1.f; }
     ms_out[i] = ms;
   }
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status acspgemm_set_trace(acspgemm_plan p, int enable) {
+  if (!p) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL plan");
+  p->trace_on = enable != 0;
+  p->trace_blocks = 0;
+  return ACSPGEMM_OK;
+}
+
+acspgemm_status acspgemm_sm_load(acspgemm_plan p, int kernel, double* per_sm_ms, int nsm, double* mpl,
+                                 int64_t* nblocks_traced) {
+  if (!p || !mpl) return set_err(ACSPGEMM_ERR_INVALID_ARG, "NULL argument");
+  if (kernel < 0 || kernel > 3) return set_err(ACSPGEMM_ERR_INVALID_ARG, "kernel must be 0..3");
+  if (!p->trace_on || p->trace_blocks <= 0 || !p->trace.p)
+    return set_err(ACSPGEMM_ERR_NOT_READY, "no traced multiply (acspgemm_set_trace before the symbolic pass)");
+  int dev = p->dev, sms = 0;
+  ACS_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  const int64_t n = p->trace_blocks;
+  std::vector<uint64_t> h((size_t)(3 * n));
+  ACS_CUDA(cudaMemcpy(h.data(), ptr<uint64_t>(p->trace) + (int64_t)kernel * 3 * n, sizeof(uint64_t) * 3 * n,
+                      cudaMemcpyDeviceToHost));
+  std::vector<double> busy((size_t)sms, 0.0);
+  int64_t traced = 0;
+  for (int64_t b = 0; b < n; ++b) {
+    const uint64_t sm = h[3 * b], t0 = h[3 * b + 1], t1 = h[3 * b + 2];
+    if (t1 == 0 || t1 < t0 || sm >= (uint64_t)sms) continue;
+    busy[(size_t)sm] += (double)(t1 - t0) * 1e-6;
+    ++traced;
+  }
+  double mx = 0.0, mn = 0.0;
+  if (traced > 0) {
+    mx = *std::max_element(busy.begin(), busy.end());
+    mn = *std::min_element(busy.begin(), busy.end());
+  }
+  *mpl = mx > 0.0 ? mn / mx : 0.0;
+  if (nblocks_traced) *nblocks_traced = traced;
+  if (per_sm_ms)
+    for (int i = 0; i < nsm && i < sms; ++i) per_sm_ms[i] = busy[(size_t)i];
   return ACSPGEMM_OK;
 }
 

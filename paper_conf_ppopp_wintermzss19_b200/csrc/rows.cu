@@ -63,6 +63,7 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const int b = blockIdx.x;
   if (a.hash_done[b] != 0) return;       // finished by an accumulator already
+  const uint64_t t_start = a.trace ? global_timer() : 0;
   const int32_t* __restrict__ bcol = a.B.col;
   const T* __restrict__ bval = reinterpret_cast<const T*>(a.B.val);
   if (tid == 0) S.flag = 0;
@@ -177,6 +178,7 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
     S.wout[w][4] = last_count;
   }
   __syncthreads();
+  if (tid == 0) trace_block(a.trace, b, t_start);
   if (tid == 0 && !S.flag) {
     emit_warp_chunks(a, b, ROWS_WARPS, S.wrow, S.wout, S.wd, S.row_first, a.rows_count);
     a.hash_done[b] = 3;

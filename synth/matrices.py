@@ -47,6 +47,27 @@ def _idx_dtype(n: int):
     return np.int32 if n < 2**31 else np.int64
 
 
+def _stable_argsort(key: np.ndarray) -> np.ndarray:
+    """np.argsort(key, kind="stable"), computed by torch's multi-threaded CPU sort when
+    torch is importable (the same permutation: a stable sort is unique)."""
+    try:
+        import torch
+    except ImportError:
+        return np.argsort(key, kind="stable")
+    return torch.sort(torch.from_numpy(np.ascontiguousarray(key)), stable=True).indices.numpy()
+
+
+def _sorted_unique(key: np.ndarray) -> np.ndarray:
+    """np.unique(key) (sorted, distinct) through a sort and a neighbour test."""
+    if key.size == 0:
+        return key
+    k = key[_stable_argsort(key)]
+    keep = np.empty(k.size, dtype=bool)
+    keep[0] = True
+    np.not_equal(k[1:], k[:-1], out=keep[1:])
+    return k[keep]
+
+
 def from_coo(rows: int, cols: int, r: np.ndarray, c: np.ndarray, v: np.ndarray,
              sum_duplicates: bool = False) -> CSR:
     """Build canonical CSR from COO triplets (sorted by (row, col))."""
@@ -54,7 +75,7 @@ def from_coo(rows: int, cols: int, r: np.ndarray, c: np.ndarray, v: np.ndarray,
     c = np.asarray(c, dtype=np.int64)
     v = np.asarray(v)
     key = r * np.int64(cols) + c
-    order = np.argsort(key, kind="stable")
+    order = _stable_argsort(key)
     key = key[order]
     v = v[order]
     if sum_duplicates and key.size:
@@ -174,7 +195,7 @@ def rmat(scale: int = 20, edge_factor: int = 16, abc=(0.45, 0.15, 0.15), seed: i
     perm = rng.permutation(n)
     src, dst = perm[src], perm[dst]
     keep = src != dst
-    key = np.unique(src[keep] * n + dst[keep])
+    key = _sorted_unique(src[keep] * n + dst[keep])
     r_, c_ = key // n, key % n
     nnz = key.size
     if values == "ones":

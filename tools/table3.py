@@ -1,7 +1,10 @@
 """Table-3-style memory report (Table 3) for the synthetic workloads:
 helper memory, chunk pool reserved (exact per-block bound, reading R8) next to the
 paper's pool estimate (L556), chunk memory used, used/output (u/o), restarts (always 0:
-the deterministic allocator never restarts) and nnz(C).  Run on a GPU box:
+the deterministic allocator never restarts), nnz(C) and the lowest multiprocessor load
+(mpL, L760/L832: min over SMs / max over SMs of the summed block time of each stage-2
+kernel that processed blocks, from acspgemm_set_trace / acspgemm_sm_load, reading R36).
+Run on a GPU box:
     python tools/table3.py > profiles/r1_table3.md
 """
 import os
@@ -22,23 +25,29 @@ def row(name, A, B, dt):
     dA = acs.DeviceCSR.from_host(A, "cuda", dt)
     dB = dA if B is A else acs.DeviceCSR.from_host(B, "cuda", dt)
     plan = acs.Plan()
+    plan.set_trace(True)
     C = plan.multiply(dA, dB)
     torch.cuda.synchronize()
     i = plan.info()
+    mpl = []
+    for k in ("hash", "rows", "esc", "esc_small"):
+        L = plan.sm_load(k)
+        if L["blocks"] > 0:
+            mpl.append(f"{k} {100 * L['mpl']:.1f} % ({L['blocks']:,})")
     used = i["chunk_elems"] * (4 + vb)
     out = i["nnz_c"] * (4 + vb)
     MB = 1e6
     line = (f"| {name} | {np.dtype(dt).name} | {i['helper_bytes'] / MB:.1f} | {i['pool_bytes'] / MB:.1f} | "
             f"{i['pool_estimate_bytes'] / MB:.1f} | {used / MB:.1f} | {100 * used / max(i['pool_bytes'], 1):.1f} % | "
-            f"{used / max(out, 1):.2f} | 0 | {i['nnz_c']:,} | {i['nchunks']:,} | {i['nshared']:,} |")
+            f"{used / max(out, 1):.2f} | 0 | {'; '.join(mpl)} | {i['nnz_c']:,} | {i['nchunks']:,} | {i['nshared']:,} |")
     print(line, flush=True)
     del C, dA, dB
     plan.close()
     torch.cuda.empty_cache()
 
 
-print("| workload | dtype | helper MB | pool MB (exact bound) | pool MB (paper estimate) | used MB | % | u/o | restarts | nnz(C) | chunks | shared rows |")
-print("|---|---|---|---|---|---|---|---|---|---|---|---|")
+print("| workload | dtype | helper MB | pool MB (reserved) | pool MB (paper estimate) | used MB | % | u/o | restarts | mpL (kernel, blocks) | nnz(C) | chunks | shared rows |")
+print("|---|---|---|---|---|---|---|---|---|---|---|---|---|")
 for cfg in ("cfg1", "cfg2", "cfg3", "cfg5"):
     A, B = config(cfg)
     row(cfg, A, B if cfg == "cfg5" else A, np.float64)
