@@ -39,6 +39,13 @@ constexpr int RADIX_BITS = ACS_RADIX_BITS;   // digit width of one radix-sort pa
 constexpr int DEFAULT_SEGMENTS = 8;          // canonical segments
 constexpr int MAX_SEGMENTS = 64;
 constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)
+// long rows (§3.4): an entry whose B row has more than PTR_LEN entries becomes
+// its own chunk (a·B_k, no sort); at most PTR_MAX such entries per block
+#ifndef ACS_PTR_LEN
+#define ACS_PTR_LEN (ACS_THREADS * ACS_ITEMS)
+#endif
+constexpr int PTR_LEN = ACS_PTR_LEN;
+constexpr int PTR_MAX = 160;
 constexpr int SEARCH_MAXP = 1024;            // Search Merge limit; longer chunk lists: dense slices (R30)
 constexpr int GIANT_SLICE = 4096;            // columns per dense-slice CTA
 constexpr int DENSE_SPAN_RATIO = 16;         // dense slices when span <= 16 x pre-merge elements

@@ -10,6 +10,12 @@
 //     (L342-L344) -> compaction scan (Alg. 3) -> completed rows go to a chunk, the
 //     last row is kept in shared memory when it is not yet complete and has at most
 //     KEEP elements (L364-L366) -> per-row counts (L362).
+// Long rows (§3.4): an entry of A whose B row has more than PTR_LEN = CAP
+// entries would be loaded and sorted without change; instead it is removed from the
+// work distribution and becomes its own chunk, a·B_k written by a coalesced streaming
+// copy (no sort), placed in the chunk order where its products belong: the iteration
+// before it stops at its position ("we break up chunks at the position of the long
+// row", L548), and the row is merged with the rest of its chunks in the merge stage.
 // Chunk allocation is deterministic (reading R8): block b writes its chunks to a
 // slot range sized from its exact product count (stage 1), so no atomics, no
 // restarts, and the chunk id (block, running number) is the global order (L430).
@@ -35,6 +41,8 @@ struct EscState {
   int kept, kofs, kept_lrow, kept_cmin, kept_cmax;  // kept row lives in the staging area
   int seq;
   int64_t wofs;
+  int stop_row;     // local row of the next long-row chunk: the current iteration ends at its
+                    // position, a complete last row below it is not kept (INT_MAX: none)
 };
 
 // Staging slot of compacted element p.  Each thread emits ITEMS consecutive elements, so
@@ -81,7 +89,7 @@ __device__ __forceinline__ void esc_tail(EscSmem<T>& S, const EscArgs& a, EscSta
   // keep the last row for the next iteration (L366) unless the block is done or the
   // row no longer fits the kept budget (reading R13: then it is written as a partial
   // chunk and merged later)
-  const bool keep = size_after > 0 && rc_last <= KEEP;
+  const bool keep = size_after > 0 && rc_last <= KEEP && rmin + lastrel >= st.stop_row;
   const int nchunk = total - (keep ? rc_last : 0);
   // compacted element p goes to staging slot stage_slot(p): [0, nchunk) is the chunk,
   // the kept row stays at [nchunk, total) for the next iteration
@@ -306,14 +314,95 @@ __device__ __forceinline__ void esc_block(EscSmem<T>& S, const EscArgs& a, const
       if (f[j]) S.row_of[run - 1] = row[j];
     }
   }
-  wd_placework(len, S.wd, S.s.scratch);
+  // long rows (§3.4): entries with B rows of more than PTR_LEN entries (at most PTR_MAX
+  // per block, in entry order) leave the work distribution; their list (entry, products
+  // before it) lives in rp_cache's storage, dead after Fetch A
+  static_assert(3 * PTR_MAX <= NPB + 1, "long-row list fits rp_cache");
+  int* ptr_e = S.rp_cache;                      // entry
+  int* ptr_p = S.rp_cache + PTR_MAX;            // products of the entries before it
+  int* ptr_n = S.rp_cache + 2 * PTR_MAX;        // its B row length
+  int np_loc = 0;
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) np_loc += len[j] > PTR_LEN;
+  int np_tot;
+  const int prank0 = block_exclusive_sum<int>(np_loc, S.s.scratch, &np_tot);
+  int prank[NNZ_PER_THREAD], plen[NNZ_PER_THREAD];
+  {
+    int r = prank0;
+#pragma unroll
+    for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+      const bool lng = len[j] > PTR_LEN;
+      prank[j] = lng && r < PTR_MAX ? r : -1;   // beyond PTR_MAX: AC-ESC as any entry
+      r += lng;
+      plen[j] = len[j];
+      if (prank[j] >= 0) len[j] = 0;
+    }
+  }
+  wd_placework(len, S.wd, S.s.scratch);          // ends with a barrier: rp_cache is free
+#pragma unroll
+  for (int j = 0; j < NNZ_PER_THREAD; ++j) {
+    if (prank[j] >= 0) {
+      const int e = tid * NNZ_PER_THREAD + j;
+      ptr_e[prank[j]] = e;
+      ptr_p[prank[j]] = S.wd[e];
+      ptr_n[prank[j]] = plen[j];
+    }
+  }
+  const int np = min(np_tot, PTR_MAX);
+  __syncthreads();
 
-  EscState st{0, 0, 0, 0, 0, 0, 0};
+  EscState st{0, 0, 0, 0, 0, 0, 0, INT_MAX};
   const int64_t pool_base = a.pool_off[b];
   const int64_t desc_base = a.desc_off[b];
-  int size = S.wd[NPB];
-  while (size > 0) {
-    const int consume = min(CAP - st.kept, size);
+  const int total_products = S.wd[NPB];
+  int size = total_products;
+  int pc = 0;                                   // next long-row entry
+  // the long-row chunks whose position has been reached: a·B_k streamed into the pool
+  auto emit_long = [&](int upto_products) {
+    while (pc < np && ptr_p[pc] <= upto_products) {
+      const int e = ptr_e[pc];
+      const int n = ptr_n[pc];
+      const int bs = S.a_bstart[e];
+      const T av = S.a_val[e];
+      const int64_t dst = pool_base + st.wofs;
+      T* pv = reinterpret_cast<T*>(a.pool_val);
+      for (int i = tid; i < n; i += THREADS) {
+        a.pool_col[dst + i] = __ldg(bcol + bs + i);
+        pv[dst + i] = av * __ldg(bval + bs + i);
+      }
+      if (tid == 0) {
+        const int grow = S.row_of[S.a_lrow[e]];
+        ChunkDesc d;
+        d.data_off = dst;
+        d.first_row = grow;
+        d.last_row = grow;
+        d.count = n;
+        d.first_count = n;
+        d.last_count = n;
+        d.flags = 0;
+        a.descs[desc_base + st.seq] = d;
+        a.row_count[grow] = n;                  // a row with other chunks is merged (count rewritten)
+      }
+      st.seq += 1;
+      st.wofs += n;
+      ++pc;
+    }
+  };
+  while (size > 0 || pc < np) {
+    const int consumed = total_products - size;
+    emit_long(consumed);
+    if (size == 0) break;
+    // stop at the next long-row chunk's position (L548); keep no complete row below it
+    int consume = min(CAP - st.kept, size);
+    st.stop_row = INT_MAX;
+    if (pc < np && ptr_p[pc] - consumed <= consume) {
+      consume = ptr_p[pc] - consumed;           // this iteration ends at the long row(s)
+      // the last row may stay (be kept) only if it is the row of the last long-row chunk
+      // emitted at this position: every chunk of a row must stay adjacent (L430)
+      int last = pc;
+      while (last + 1 < np && ptr_p[last + 1] == ptr_p[pc]) ++last;
+      st.stop_row = S.a_lrow[ptr_e[last]];
+    }
     // the kept row sits in the staging area, which the new values overwrite: pull it
     // into registers first (receivework's barriers order this before the writes)
     int kc[KEEP_PER_THREAD];
@@ -384,6 +473,7 @@ __device__ __forceinline__ void esc_block(EscSmem<T>& S, const EscArgs& a, const
                                  pool_base, desc_base);
     size = size_after;
   }
+  emit_long(INT_MAX);
   if (tid == 0) {
     a.nchunks[b] = st.seq;
     a.used[b] = (int32_t)st.wofs;

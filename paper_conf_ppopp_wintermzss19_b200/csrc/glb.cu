@@ -134,6 +134,7 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
     const int64_t nzb = s_nz[s] + (b - s_base[s]) * NPB;
     const int64_t nze = min(nzb + (int64_t)NPB, s_nz[s + 1]);
     int64_t sum = 0, waves = 0;
+    int nlong = 0;                            // long-row chunks (§3.4): one chunk + one split each
     // all of the block's column loads first (NPB / 32 per lane), then the B row gathers
     constexpr int PER_LANE = NPB / 32;
     int k[PER_LANE];
@@ -148,12 +149,14 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
         const int len = brp[k[j] + 1] - brp[k[j]];
         sum += len;
         waves += (len + 31) >> 5;
+        nlong += len > PTR_LEN;
       }
     }
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) {
       sum += __shfl_xor_sync(0xffffffffu, sum, d);
       waves += __shfl_xor_sync(0xffffffffu, waves, d);
+      nlong += __shfl_xor_sync(0xffffffffu, nlong, d);
     }
     int hok = 0;
     if (hash_ok && sum > 0 && 2 * sum >= 32 * waves) {
@@ -197,7 +200,8 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
       if (hok) atomicAdd(&s_cand, 1);
       products[b] = sum;
       // the accumulators (R31, R33) emit up to one chunk per warp
-      slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)ACC_MAX_WARPS) : 0;
+      slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)ACC_MAX_WARPS) +
+                               2 * (int64_t)min(nlong, PTR_MAX) : 0;
       nz_begin[b] = (int32_t)nzb;
       nz_end[b] = (int32_t)nze;
     }

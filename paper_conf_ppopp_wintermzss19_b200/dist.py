@@ -131,3 +131,69 @@ def dist_multiply(A, B, group=None, S: int = S_DEFAULT,
         dev = torch.device("cuda", torch.cuda.current_device())
     offs = gather_offsets(nnz, rows, group, dev)
     return C, offs[g], offs
+
+
+def allgather_csr_pieces(piece, rows_total: int, cols: int, group=None):
+    """The one exchange step of the distributed Galerkin product: every
+    rank's CSR piece (row_ptr, col, val; numpy or torch) -> the concatenated matrix on
+    every rank.  NCCL: device tensors padded to the largest piece; gloo: CPU objects."""
+    import numpy as np
+    from .api import DeviceCSR
+    ws = dist.get_world_size(group)
+    if dist.get_backend(group) != "nccl":
+        allp = [None] * ws
+        to_np = lambda t: t.cpu().numpy() if hasattr(t, "cpu") else np.asarray(t)   # noqa: E731
+        dist.all_gather_object(allp, tuple(to_np(t) for t in piece), group=group)
+        rp, col, val = concat_pieces(allp)
+        return rp, col, val
+    dev = torch.device("cuda", torch.cuda.current_device())
+    rp, col, val = piece
+    sizes = torch.tensor([rp.numel() - 1, col.numel()], dtype=torch.int64, device=dev)
+    alls = [torch.zeros_like(sizes) for _ in range(ws)]
+    dist.all_gather(alls, sizes, group=group)
+    mr = max(int(a[0]) for a in alls)
+    mn = max(int(a[1]) for a in alls)
+    def gather(t, n, dtype):
+        buf = torch.zeros(n, dtype=dtype, device=dev)
+        buf[:t.numel()] = t
+        outs = [torch.empty_like(buf) for _ in range(ws)]
+        dist.all_gather(outs, buf, group=group)
+        return outs
+    rps = gather(rp.to(torch.int64), mr + 1, torch.int64)
+    cols = gather(col, max(mn, 1), col.dtype)
+    vals = gather(val, max(mn, 1), val.dtype)
+    out_rp, out_c, out_v, off = [torch.zeros(1, dtype=torch.int64, device=dev)], [], [], 0
+    for g in range(ws):
+        r, n = int(alls[g][0]), int(alls[g][1])
+        out_rp.append(rps[g][1:r + 1] - rps[g][0] + off)
+        out_c.append(cols[g][:n])
+        out_v.append(vals[g][:n])
+        off += n
+    full_rp = torch.cat(out_rp).to(torch.int32)
+    assert full_rp.numel() == rows_total + 1
+    return DeviceCSR(rows_total, cols, full_rp.contiguous(), torch.cat(out_c).contiguous(),
+                     torch.cat(out_v).contiguous())
+
+
+def dist_rap(R, A, P, group=None, S: int = S_DEFAULT, local_multiply: Optional[Callable] = None):
+    """Galerkin product R·(A·P) over the process group.
+
+    Step 1: each rank multiplies its canonical segments of A's fine rows with P (no
+    exchange: P is replicated).  Step 2: one all-gather of the A·P pieces -- R's coarse
+    rows reach fine rows of every segment.  Step 3: each rank multiplies its canonical
+    segments of R with the gathered A·P.  Both products use canonical segments, so the
+    concatenated result is byte-identical to the 1-GPU R·(A·P) (acspgemm_rap).
+    Returns (this rank's piece of R·A·P, its (row, nnz) offset, all offsets)."""
+    AP_piece, _, _ = dist_multiply(A, P, group, S, local_multiply)
+    AP = allgather_csr_pieces((AP_piece.row_ptr, AP_piece.col, AP_piece.val), A.rows, P.cols, group)
+    if isinstance(AP, tuple):                      # gloo: the gathered A·P arrives on the host
+        rp, col, val = AP
+        if local_multiply is None:                 # the CUDA path: back to the device
+            from .api import DeviceCSR
+            dev = torch.device("cuda", torch.cuda.current_device())
+            AP = DeviceCSR(A.rows, P.cols, torch.from_numpy(rp.astype("int32")).to(dev),
+                           torch.from_numpy(col).to(dev), torch.from_numpy(val).to(dev))
+        else:                                      # a CPU stand-in multiply (tests)
+            from types import SimpleNamespace
+            AP = SimpleNamespace(rows=A.rows, cols=P.cols, row_ptr=rp, col=col, val=val)
+    return dist_multiply(R, AP, group, S, local_multiply)

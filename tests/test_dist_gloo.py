@@ -91,3 +91,50 @@ def test_rank_segments_and_offsets():
         assert canonical_segments_host(rp, 8) == alg.canonical_segments(rp, 8)
     seg = [0, 10, 25, 40]
     assert adist.local_segment_rows(seg, 1, 3) == [0, 15, 30]
+
+
+def _rap_worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import oracle
+    from paper_conf_ppopp_wintermzss19_b200 import dist as adist
+    from synth import aggregation_prolongator, poisson3d_7pt, transpose
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    try:
+        n = 8
+        A = poisson3d_7pt(n)
+        P = aggregation_prolongator(n)
+        R = transpose(P)
+
+        def local(A_, B_, seg, s0, s1):
+            return oracle.gustavson(A_, B_, row_begin=int(seg[s0]), row_end=int(seg[s1]))
+
+        C, _, offs = adist.dist_rap(R, A, P, local_multiply=local)
+        pieces = [None] * world
+        dist.all_gather_object(pieces, (C.row_ptr, C.col, C.val))
+        if rank == 0:
+            rp, col, val = adist.concat_pieces(pieces)
+            A4 = poisson3d_7pt(n // 2)       # R·A·P = 4·A7(n/2) (the closed form of the oracle tests)
+            ok = ((rp == A4.row_ptr).all() and (col == A4.col).all() and (val == 4 * A4.val).all())
+            q.put(bool(ok))
+        else:
+            q.put(True)
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_dist_rap_gloo(world):
+    """Distributed Galerkin product: A·P per rank, one all-gather of the
+    A·P pieces, R·(A·P) per rank; the concatenation equals 4·A7(n/2) exactly."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rap_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    assert all(p.exitcode == 0 for p in procs)
+    assert all(res), res

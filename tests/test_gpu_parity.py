@@ -402,3 +402,51 @@ def test_64bit_sort_words(cuda_available):
     cols = np.concatenate([np.sort(rng.choice(ncols, 4, replace=False)) for _ in range(K)])
     B = from_coo(K, ncols, rows, cols, rng.integers(-3, 4, rows.size).astype(np.float64))
     assert_parity(A, B, np.float64, exact=True, oracle_threads=1)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_long_row_chunks(dt, cuda_available):
+    """§3.4 long rows (L546-L548): entries whose B row has more than CAP = 2048 entries
+    become their own chunk (a·B_k, no sort) placed where their products belong.  Rows
+    made of one long entry (C row = a·B_k, no merge), long entries first / in the middle /
+    last among short ones, several per row, rows of only long entries, long entries at
+    block boundaries, and a block with more long entries than PTR_MAX (the rest go
+    through AC-ESC).  Integer values: exact; U(-1,1): within tolerance."""
+    rng = np.random.default_rng(21)
+    nb, ncols = 400, 6000
+    blen = rng.integers(5, 60, nb)
+    blen[rng.choice(nb, 60, replace=False)] = rng.integers(2049, 5000, 60)   # long B rows
+    long_rows = np.flatnonzero(blen > 2048)
+    short_rows = np.flatnonzero(blen <= 2048)
+    r, c = [], []
+    for i in range(1200):
+        kind = i % 6
+        if kind == 0:
+            k = [rng.choice(long_rows)]                                   # a single long entry
+        elif kind == 1:
+            k = list(rng.choice(short_rows, 5, replace=False)) + [rng.choice(long_rows)]
+        elif kind == 2:
+            k = list(rng.choice(long_rows, 3, replace=False))              # only long entries
+        elif kind == 3:
+            k = list(rng.choice(short_rows, 8, replace=False))
+        else:
+            k = list(rng.choice(short_rows, 6, replace=False)) + list(rng.choice(long_rows, 2, replace=False))
+        k = np.unique(k)
+        r += [i] * len(k)
+        c += k.tolist()
+    # rows 1200..1399: 200 consecutive single long entries (> PTR_MAX = 160 in a block)
+    for i in range(1200, 1400):
+        r.append(i)
+        c.append(int(long_rows[i % len(long_rows)]))
+    rr, cc = np.array(r), np.array(c)
+    for values in ("int", "uniform"):
+        if values == "int":
+            va = rng.integers(1, 4, rr.size) * rng.choice([-1.0, 1.0], rr.size)
+        else:
+            va = rng.uniform(-1, 1, rr.size)
+        A = from_coo(1400, nb, rr, cc, va)
+        rows_b = np.repeat(np.arange(nb), blen)
+        cols_b = np.concatenate([np.sort(rng.choice(ncols, L, replace=False)) for L in blen])
+        vb = rng.integers(-3, 4, rows_b.size).astype(np.float64) if values == "int" else rng.uniform(-1, 1, rows_b.size)
+        B = from_coo(nb, ncols, rows_b, cols_b, vb)
+        assert_parity(A, B, dt, exact=(values == "int"))
