@@ -100,7 +100,6 @@ struct MergeState {
   int64_t* scan_tmp;
 };
 void launch_gather_chunks(const MergeState& m, cudaStream_t st);
-void launch_find_shared(const MergeState& m, int64_t* total_shared_dev, cudaStream_t st);
 
 struct MergeLists {
   int64_t nshared;
@@ -119,7 +118,8 @@ struct MergeLists {
   int32_t* group_start;          // [max groups + 1]
   int64_t* scan_tmp;
 };
-void launch_classify(const MergeLists& L, cudaStream_t st);
+// shared rows, their kinds and merge offsets in one pass (lists sized by m.max_chunks)
+void launch_find_shared(const MergeState& m, const MergeLists& L, int64_t* total_shared_dev, cudaStream_t st);
 void launch_multi_groups(const MergeLists& L, int64_t nmulti, int64_t ngroups, cudaStream_t st);
 
 struct MergeArgs {

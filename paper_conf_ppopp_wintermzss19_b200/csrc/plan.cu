@@ -430,11 +430,36 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ms.shared = ptr<SharedRow>(p->shared);
   ms.pool_col = ptr<int32_t>(p->pool_col);
   ms.scan_tmp = ptr<int64_t>(p->scan_tmp);
+  // merge lists sized by the chunk bound: shared rows, their kinds and merge offsets
+  // are found in one pass, and one read-back serves MCC
+  ACS_ENSURE(p->kflag, sizeof(int32_t) * std::max<int64_t>(slots, 1));
+  ACS_ENSURE(p->lmulti, sizeof(int32_t) * std::max<int64_t>(slots, 1));
+  ACS_ENSURE(p->lpath, sizeof(int32_t) * std::max<int64_t>(slots, 1));
+  ACS_ENSURE(p->lsearch, sizeof(int32_t) * std::max<int64_t>(slots, 1));
+  ACS_ENSURE(p->lpair, sizeof(int32_t) * std::max<int64_t>(slots, 1));
+  ACS_ENSURE(p->lgiant, sizeof(int32_t) * std::max<int64_t>(slots, 1));
+  ACS_ENSURE(p->mtscan, sizeof(int64_t) * std::max<int64_t>(slots, 1));
+  MergeLists L;
+  L.nshared = 0;
+  L.shared = ptr<SharedRow>(p->shared);
+  L.kind_flag = ptr<int32_t>(p->kflag);
+  L.kind_pos = nullptr;
+  L.multi_idx = ptr<int32_t>(p->lmulti);
+  L.path_idx = ptr<int32_t>(p->lpath);
+  L.search_idx = ptr<int32_t>(p->lsearch);
+  L.pair_idx = ptr<int32_t>(p->lpair);
+  L.giant_idx = ptr<int32_t>(p->lgiant);
+  L.counts_dev = scal + 8;
+  L.merge_total_scan = ptr<int64_t>(p->mtscan);
+  L.multi_scan = nullptr;
+  L.group_of = nullptr;
+  L.group_start = nullptr;
+  L.scan_tmp = ptr<int64_t>(p->scan_tmp);
   launch_gather_chunks(ms, st);
-  launch_find_shared(ms, scal + 4, st);
-  tl_launches += 1 + (slots > 0 ? 5 : 0);
+  launch_find_shared(ms, L, scal + 4, st);
+  tl_launches += 1 + (slots > 0 ? 11 : 0);
   ACS_CUDA(cudaGetLastError());
-  if ((s = sync_read(p, scal + 2, 6, st)) != ACSPGEMM_OK) return s;
+  if ((s = sync_read(p, scal + 2, 12, st)) != ACSPGEMM_OK) return s;
   p->info.nrow_blocks = p->h_scal[0];
   p->info.nhash_blocks = p->h_scal[4];
   p->info.ndict_blocks = p->h_scal[5];
@@ -447,36 +472,12 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   const int64_t nsh = p->nshared;
   int64_t nmulti = 0, npath = 0, nsearch = 0, npair = 0, merge_total = 0, ngroups = 0, ngiant = 0;
   if (nsh > 0) {
-    ACS_ENSURE(p->kflag, sizeof(int32_t) * nsh);
-    ACS_ENSURE(p->kpos, sizeof(int64_t) * nsh);
-    ACS_ENSURE(p->lmulti, sizeof(int32_t) * nsh);
-    ACS_ENSURE(p->lpath, sizeof(int32_t) * nsh);
-    ACS_ENSURE(p->lsearch, sizeof(int32_t) * nsh);
-    ACS_ENSURE(p->lpair, sizeof(int32_t) * nsh);
-    ACS_ENSURE(p->lgiant, sizeof(int32_t) * nsh);
-    ACS_ENSURE(p->mtscan, sizeof(int64_t) * nsh);
     ACS_ENSURE(p->mscan, sizeof(int64_t) * nsh);
     ACS_ENSURE(p->group_of, sizeof(int32_t) * nsh);
-    MergeLists L;
     L.nshared = nsh;
-    L.shared = ptr<SharedRow>(p->shared);
-    L.kind_flag = ptr<int32_t>(p->kflag);
-    L.kind_pos = ptr<int64_t>(p->kpos);
-    L.multi_idx = ptr<int32_t>(p->lmulti);
-    L.path_idx = ptr<int32_t>(p->lpath);
-    L.search_idx = ptr<int32_t>(p->lsearch);
-    L.pair_idx = ptr<int32_t>(p->lpair);
-    L.giant_idx = ptr<int32_t>(p->lgiant);
-    L.counts_dev = scal + 8;
-    L.merge_total_scan = ptr<int64_t>(p->mtscan);
     L.multi_scan = ptr<int64_t>(p->mscan);
     L.group_of = ptr<int32_t>(p->group_of);
-    L.group_start = nullptr;
-    L.scan_tmp = ptr<int64_t>(p->scan_tmp);
-    launch_classify(L, st);
-    tl_launches += 5 * 5 + 1 + 3 + 1;
-    ACS_CUDA(cudaGetLastError());
-    if ((s = sync_read(p, scal + 8, 6, st)) != ACSPGEMM_OK) return s;
+    for (int i = 0; i < 6; ++i) p->h_scal[i] = p->h_scal[6 + i];   // the class counts (scal + 8 ..)
     nmulti = p->h_scal[0];
     npath = p->h_scal[1];
     nsearch = p->h_scal[2];

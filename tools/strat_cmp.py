@@ -46,7 +46,7 @@ for strat in strats:
     info = plan.info()
     med = {k: round(float(np.median([s[k] for s in st_all])), 3) for k in st_all[0]}
     print(json.dumps({"cfg": cfg, "dtype": str(np.dtype(dt)), "strategy": strat, "ms": e0.elapsed_time(e1) / reps,
-                      "stages": med, "nblocks": info["nblocks"], "nspa": info["nspa_blocks"],
+                      "stages": med, "nblocks": info["nblocks"], 
                       "ndict": info["ndict_blocks"], "nhash": info["nhash_blocks"], "nrows": info["nrow_blocks"],
                       "sha": digests[strat]}), flush=True)
     plan.close()
