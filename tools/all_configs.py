@@ -1,3 +1,4 @@
+"""Every BASELINE config: ms, GFLOPS, per-stage times, path counters (one JSON line each).  usage: python tools/all_configs.py [cfg1,cfg2,cfg3,cfg5,cfg4]"""
 import sys, os, time, json
 sys.path.insert(0, os.getcwd())
 import numpy as np, torch

@@ -1,4 +1,4 @@
-"""Per-source-line instruction / stall-sample shares from an ncu report (source page)."""
+"""Per-source-line instruction / stall-sample shares from an ncu report (source page).  usage: python tools/ncu_lines.py REPORT.ncu-rep [N]"""
 import csv, subprocess, sys
 rep, n = sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 40
 txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],

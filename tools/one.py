@@ -1,4 +1,4 @@
-"""Two multiplies of one config (for ncu captures).  usage: python scratch/one.py CFG [f64|f32] [strategy]"""
+"""Two multiplies of one config (for ncu captures).  usage: python tools/one.py CFG [f64|f32] [strategy]"""
 import sys, os
 sys.path.insert(0, os.getcwd())
 import numpy as np, torch, paper_conf_ppopp_wintermzss19_b200 as acs
