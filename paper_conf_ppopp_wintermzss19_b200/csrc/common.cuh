@@ -48,7 +48,10 @@ constexpr int PTR_LEN = ACS_PTR_LEN;
 constexpr int PTR_MAX = 160;
 constexpr int SEARCH_MAXP = 1024;            // Search Merge limit; longer chunk lists: dense slices (R30)
 constexpr int GIANT_SLICE = 4096;            // columns per dense-slice CTA
-constexpr int DENSE_SPAN_RATIO = 16;         // dense slices when span <= 16 x pre-merge elements
+#ifndef ACS_DENSE_SPAN_RATIO
+#define ACS_DENSE_SPAN_RATIO 16
+#endif
+constexpr int DENSE_SPAN_RATIO = ACS_DENSE_SPAN_RATIO;  // dense slices when span <= 16 x pre-merge elements
 #ifndef ACS_PAIR_MAX
 #define ACS_PAIR_MAX 512
 #endif

@@ -42,7 +42,9 @@ struct EscState {
   int seq;
   int64_t wofs;
   int stop_row;     // local row of the next long-row chunk: the current iteration ends at its
-                    // position, a complete last row below it is not kept (INT_MAX: none)
+                    // position, a complete last row below it is not kept (INT_MIN: none)
+  bool keep_ok;     // the block's rows average at most CAP/2 products (reading R38): keeping
+                    // the last row (L366) can spare a merge; longer rows span iterations anyway
 };
 
 // Staging slot of compacted element p.  Each thread emits ITEMS consecutive elements, so
@@ -89,7 +91,7 @@ __device__ __forceinline__ void esc_tail(EscSmem<T>& S, const EscArgs& a, EscSta
   // keep the last row for the next iteration (L366) unless the block is done or the
   // row no longer fits the kept budget (reading R13: then it is written as a partial
   // chunk and merged later)
-  const bool keep = size_after > 0 && rc_last <= KEEP && rmin + lastrel >= st.stop_row;
+  const bool keep = st.keep_ok && size_after > 0 && rc_last <= KEEP && rmin + lastrel >= st.stop_row;
   const int nchunk = total - (keep ? rc_last : 0);
   // compacted element p goes to staging slot stage_slot(p): [0, nchunk) is the chunk,
   // the kept row stays at [nchunk, total) for the next iteration
@@ -351,10 +353,11 @@ __device__ __forceinline__ void esc_block(EscSmem<T>& S, const EscArgs& a, const
   const int np = min(np_tot, PTR_MAX);
   __syncthreads();
 
-  EscState st{0, 0, 0, 0, 0, 0, 0, INT_MAX};
+  EscState st{0, 0, 0, 0, 0, 0, 0, INT_MIN, true};
   const int64_t pool_base = a.pool_off[b];
   const int64_t desc_base = a.desc_off[b];
   const int total_products = S.wd[NPB];
+  st.keep_ok = (int64_t)total_products <= (int64_t)(CAP / 2) * tot;
   int size = total_products;
   int pc = 0;                                   // next long-row entry
   // the long-row chunks whose position has been reached: a·B_k streamed into the pool
@@ -394,7 +397,7 @@ __device__ __forceinline__ void esc_block(EscSmem<T>& S, const EscArgs& a, const
     if (size == 0) break;
     // stop at the next long-row chunk's position (L548); keep no complete row below it
     int consume = min(CAP - st.kept, size);
-    st.stop_row = INT_MAX;
+    st.stop_row = INT_MIN;
     if (pc < np && ptr_p[pc] - consumed <= consume) {
       consume = ptr_p[pc] - consumed;           // this iteration ends at the long row(s)
       // the last row may stay (be kept) only if it is the row of the last long-row chunk

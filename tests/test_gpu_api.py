@@ -225,3 +225,36 @@ def test_multiply_host_rectangular_capacity(cuda_available):
     assert (np.abs(val - ref.val) <= 1e-12 * ref.absval).all()
     # the plan's own segmentation is restored afterwards
     check(plan.multiply(dev(A), dev(B)), A, B)
+
+
+def test_sm_load_trace(cuda_available):
+    """Table 3's lowest multiprocessor load (mpL, L760): with tracing on, every block a
+    stage-2 kernel processed is recorded once (SM id, start, end); mpL is in (0, 1] for
+    a kernel that ran on every SM, the per-SM busy times are non-negative, tracing
+    changes no result, and an untraced plan reports NOT_READY."""
+    import paper_conf_ppopp_wintermzss19_b200 as p
+    from synth import poisson3d_27pt, power_law_csr
+    A = poisson3d_27pt(40)
+    dA = p.DeviceCSR.from_host(A, "cuda")
+    plan = p.Plan()
+    ref = plan.multiply(dA, dA)
+    with pytest.raises(p.AcspgemmError):
+        plan.sm_load("hash")
+    plan.set_trace(True)
+    C = plan.multiply(dA, dA)
+    torch.cuda.synchronize()
+    assert all(torch.equal(x, y) for x, y in ((C.row_ptr, ref.row_ptr), (C.col, ref.col), (C.val, ref.val)))
+    info = plan.info()
+    L = plan.sm_load("hash")
+    assert L["blocks"] == info["nhash_blocks"] > 0
+    assert 0.0 < L["mpl"] <= 1.0 and min(L["per_sm_ms"]) >= 0.0
+    B = power_law_csr(3000, 3000, mean_len=12, alpha=1.3, max_len=800, seed=2)
+    dB = p.DeviceCSR.from_host(B, "cuda")
+    plan.multiply(dB, dB)
+    E = plan.sm_load("esc")
+    assert E["blocks"] > 0 and 0.0 <= E["mpl"] <= 1.0
+    plan.set_trace(False)
+    plan.multiply(dB, dB)
+    with pytest.raises(p.AcspgemmError):
+        plan.sm_load("esc")
+    plan.close()
