@@ -62,6 +62,25 @@ def main():
     Ag = from_coo(3, n_b, [0] * n_b + [1, 1], list(range(n_b)) + [5, 9], rng.uniform(-1, 1, n_b + 2))
     Bg = random_rowlen_csr(n_b, 100000, np.full(n_b, 32), seed=18, values="uniform")
     case("giant row (dense slices)", Ag, Bg, np.float64)
+    # long B rows (> CAP entries): long-row chunks (R35) between short entries
+    nb = 120
+    blen = rng.integers(5, 40, nb)
+    blen[::7] = rng.integers(2100, 3000, len(blen[::7]))
+    Bl = random_rowlen_csr(nb, 4000, blen, seed=21)
+    Al = random_rowlen_csr(600, nb, rng.integers(1, 10, 600), seed=22)
+    case("long B rows (long-row chunks)", Al, Bl, np.float64)
+    # LP-like: rows of ~1,600 products (no kept row, R38; two-chunk rows > 512: Multi Merge)
+    from synth import lp_like
+    Alp, Atp = lp_like(rows_log2=11, cols_log2=13, per_col=20, seed=7)
+    case("LP-like (Multi Merge)", Alp, Atp, np.float64)
+    plan = acs.Plan()
+    plan.set_trace(True)
+    dT = acs.DeviceCSR.from_host(s27, "cuda")
+    plan.multiply(dT, dT)
+    torch.cuda.synchronize()
+    assert plan.sm_load("hash")["blocks"] > 0
+    plan.close()
+    print("traced multiply (mpL) ok", flush=True)
     Ar, Br = random_csr(800, 700, 0.02, seed=1), random_csr(700, 900, 0.02, seed=2)
     case("random", Ar, Br, np.float32)
     Ae = from_coo(4, 6, [], [], [])
