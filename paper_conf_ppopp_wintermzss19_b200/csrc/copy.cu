@@ -86,6 +86,21 @@ void launch_read_back(const void* src, void* mapped_dst, int nbytes, cudaStream_
                                                    static_cast<uint32_t*>(mapped_dst), nw);
 }
 
+__global__ void k_read_back2(const uint32_t* __restrict__ src1, volatile uint32_t* dst1, int n1,
+                             const uint32_t* __restrict__ src2, volatile uint32_t* dst2, int n2) {
+  const int i = threadIdx.x;
+  if (i < n1) dst1[i] = src1[i];
+  if (i < n2) dst2[i] = src2[i];
+}
+
+void launch_read_back2(const void* src1, void* dst1, int nbytes1, const void* src2, void* dst2, int nbytes2,
+                       cudaStream_t st) {
+  const int n1 = (nbytes1 + 3) / 4, n2 = (nbytes2 + 3) / 4, nw = n1 > n2 ? n1 : n2;
+  k_read_back2<<<1, 32 * ((nw + 31) / 32), 0, st>>>(static_cast<const uint32_t*>(src1), static_cast<uint32_t*>(dst1),
+                                                    n1, static_cast<const uint32_t*>(src2),
+                                                    static_cast<uint32_t*>(dst2), n2);
+}
+
 __global__ void k_copy_offset(int32_t* __restrict__ dst, const int32_t* __restrict__ src, int64_t n, int32_t off) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     dst[i] = src[i] + off;

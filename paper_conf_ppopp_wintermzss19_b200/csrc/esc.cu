@@ -512,31 +512,6 @@ __global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
   }
 }
 
-// warp-aggregated append of b to list (any order)
-__device__ __forceinline__ void list_append(bool need, int b, int32_t* list, int64_t* count) {
-  const unsigned m = __ballot_sync(0xffffffffu, need);
-  if (!m) return;
-  int base = 0;
-  if ((threadIdx.x & 31) == __ffs(m) - 1)
-    base = (int)atomicAdd(reinterpret_cast<unsigned long long*>(count), (unsigned long long)__popc(m));
-  base = __shfl_sync(0xffffffffu, base, __ffs(m) - 1);
-  if (need) list[base + __popc(m & ((1u << (threadIdx.x & 31)) - 1u))] = b;
-}
-
-// lists of the blocks k_hash left to AC-ESC: blocks of at most CAP_SMALL products go to
-// the small-tile AC-ESC (one iteration of a 512-slot tile, reading R32), the rest here
-__global__ void k_esc_list(EscArgs a) {
-  const int b = blockIdx.x * blockDim.x + threadIdx.x;
-  const bool need = b < a.nblocks && !a.hash_done[b];
-  const bool small = need && a.esc_list_small && a.blk_products[b] <= CAP_SMALL;
-  list_append(need && !small, b, a.esc_list, a.esc_count);
-  list_append(small, b, a.esc_list_small, a.esc_count_small);
-}
-
-void launch_esc_lists(const EscArgs& a, cudaStream_t st) {
-  if (a.nblocks > 0 && a.hash_done) k_esc_list<<<(a.nblocks + 255) / 256, 256, 0, st>>>(a);
-}
-
 template <typename T>
 static void launch_esc_t(const EscArgs& a, cudaStream_t st) {
   const size_t smem = sizeof(EscSmem<T>);

@@ -16,9 +16,12 @@ namespace acs {
 constexpr int SEG_STRIDE = MAX_SEGMENTS + 1;
 
 __global__ void k_segments(const int32_t* __restrict__ rp, int64_t rows, int nseg, SegRows explicit_rows,
-                           int64_t* __restrict__ seg, int32_t* __restrict__ nblocks) {
+                           int64_t* __restrict__ seg, int32_t* __restrict__ nblocks, ZeroList zero) {
   __shared__ int64_t s_rows[SEG_STRIDE], s_nz[SEG_STRIDE];
   const int s = threadIdx.x;
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+    for (int j = s; j < zero.n[i]; j += blockDim.x) zero.p[i][j] = 0;
   const int64_t base = rp[0];
   const int64_t nnz = (int64_t)rp[rows] - base;
   if (s <= nseg) {
@@ -56,13 +59,13 @@ __global__ void k_segments(const int32_t* __restrict__ rp, int64_t rows, int nse
 }
 
 void launch_segments(const CsrView& A, int nseg, const SegRows& explicit_rows, int64_t* seg,
-                     int32_t* nblocks_dev, cudaStream_t st) {
-  k_segments<<<1, 128, 0, st>>>(A.row_ptr, A.rows, nseg, explicit_rows, seg, nblocks_dev);
+                     int32_t* nblocks_dev, cudaStream_t st, const ZeroList& zero) {
+  k_segments<<<1, 128, 0, st>>>(A.row_ptr, A.rows, nseg, explicit_rows, seg, nblocks_dev, zero);
 }
 
 // Alg. 1: one thread per row of A.  Reading R4: rows with a == b are skipped.
 __global__ void k_glb(const int32_t* __restrict__ rp, int64_t rows, int nseg, const int64_t* __restrict__ seg,
-                      int32_t* __restrict__ block_row_starts) {
+                      int32_t* __restrict__ block_row_starts, int32_t* __restrict__ row_count) {
   __shared__ int64_t s_rows[SEG_STRIDE], s_nz[SEG_STRIDE], s_base[SEG_STRIDE];
   for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
     s_rows[i] = seg[i];
@@ -72,6 +75,7 @@ __global__ void k_glb(const int32_t* __restrict__ rp, int64_t rows, int nseg, co
   __syncthreads();
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (tid >= rows) return;
+  if (row_count) row_count[tid] = 0;
   const int64_t a0 = rp[tid], b0 = rp[tid + 1];
   if (a0 == b0) return;
   int s = 0;                                   // segment holding row tid
@@ -85,11 +89,12 @@ __global__ void k_glb(const int32_t* __restrict__ rp, int64_t rows, int nseg, co
   }
 }
 
-void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* brs, int64_t max_blocks, cudaStream_t st) {
+void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* brs, int64_t max_blocks, cudaStream_t st,
+                int32_t* row_count) {
   (void)max_blocks;
   if (A.rows == 0) return;
   const int T = 256;
-  k_glb<<<(unsigned)((A.rows + T - 1) / T), T, 0, st>>>(A.row_ptr, A.rows, nseg, seg, brs);
+  k_glb<<<(unsigned)((A.rows + T - 1) / T), T, 0, st>>>(A.row_ptr, A.rows, nseg, seg, brs, row_count);
 }
 
 // Per block: nonzero range and the exact product count sum_p len(B_row(A.col[p])),
@@ -112,7 +117,7 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
                                int64_t max_blocks, int32_t* __restrict__ nz_begin, int32_t* __restrict__ nz_end,
                                int64_t* __restrict__ products, int64_t* __restrict__ slots,
                                int32_t* __restrict__ hash_ok, int64_t* __restrict__ ncand,
-                               int64_t* __restrict__ max_products) {
+                               int64_t* __restrict__ max_products, int64_t* __restrict__ nblocks_out) {
   __shared__ int64_t s_nz[SEG_STRIDE], s_base[SEG_STRIDE];
   __shared__ int s_cand;
   for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
@@ -124,6 +129,7 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
   const int64_t b = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   const int nblocks = *nblocks_dev;
+  if (nblocks_out && blockIdx.x == 0 && threadIdx.x == 0) *nblocks_out = nblocks;
   if (b < max_blocks && b >= nblocks && lane == 0) {
     products[b] = 0; slots[b] = 0; nz_begin[b] = 0; nz_end[b] = 0;
     if (hash_ok) hash_ok[b] = 0;
@@ -214,12 +220,12 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
 void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* nzb, int32_t* nze,
                          int64_t* products, int64_t* slots, int32_t* hash_ok, int64_t* ncand,
-                         int64_t* max_products, cudaStream_t st) {
+                         int64_t* max_products, int64_t* nblocks_out, cudaStream_t st) {
   if (max_blocks == 0) return;
   const int T = 256, WPB = T / 32;
   k_block_bounds<<<(unsigned)((max_blocks + WPB - 1) / WPB), T, 0, st>>>(
       A.row_ptr, A.col, B.row_ptr, B.col, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots, hash_ok,
-      ncand, max_products);
+      ncand, max_products, nblocks_out);
 }
 
 // Canonical-CSR check (reading R3): row_ptr monotone, columns strictly increasing and

@@ -20,21 +20,30 @@ struct SegRows {
   int32_t n;
   int64_t r[MAX_SEGMENTS + 1];
 };
-// Writes seg tables to `seg` (device, int64[4*(MAX_SEGMENTS+1)]): rows | nz | block base.
+// Device words the first kernel of a multiply zeroes (counters of the later stages), so
+// that no memset launch is needed: ZeroList::p[i][0 .. n[i]) = 0.
+struct ZeroList {
+  int64_t* p[4];
+  int32_t n[4];
+};
+// Writes seg tables to `seg` (device, int64[4*(MAX_SEGMENTS+1)]): rows | nz | block base;
+// also zeroes `zero`.
 void launch_segments(const CsrView& A, int nseg, const SegRows& explicit_rows,
-                     int64_t* seg, int32_t* nblocks_dev, cudaStream_t st);
+                     int64_t* seg, int32_t* nblocks_dev, cudaStream_t st, const ZeroList& zero = ZeroList{});
+// row_count (nullable): zeroed, one word per row of A
 void launch_glb(const CsrView& A, int nseg, const int64_t* seg, int32_t* block_row_starts,
-                int64_t max_blocks, cudaStream_t st);
+                int64_t max_blocks, cudaStream_t st, int32_t* row_count = nullptr);
 void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* blk_nz_begin,
                          int32_t* blk_nz_end, int64_t* blk_products, int64_t* blk_slots,
                          int32_t* blk_hash_ok /* nullable: hash-accumulator candidates (R31) */,
                          int64_t* ncand /* nullable: their count (zeroed by the caller) */,
                          int64_t* max_products /* atomicMax of block products > INT_MAX (zeroed) */,
-                         cudaStream_t st);
+                         int64_t* nblocks_out /* nullable: the block count as int64 */, cudaStream_t st);
 
 // ---- device-wide exclusive scan (scan.cu) --------------------------------------
-// out[i] = sum_{j<i} in[j] for i < n, total -> *total_dev.  tmp needs scan_tmp_elems(n).
+// out[i] = sum_{j<i} in[j] for i < n, total -> *total_dev.  tmp needs scan_tmp_elems(n)
+// words, all zero before the first scan; every scan leaves them zero again.
 int64_t scan_tmp_elems(int64_t n);
 void launch_scan_i64(const int64_t* in, int64_t* out, int64_t n, int64_t* total_dev, int64_t* tmp, cudaStream_t st);
 void launch_scan_i32(const int32_t* in, int64_t* out, int64_t n, int64_t* total_dev, int64_t* tmp, cudaStream_t st);
@@ -70,17 +79,17 @@ struct EscArgs {
   int32_t* esc_list_small;      // adaptive: left blocks of <= CAP_SMALL products [nblocks]
   int64_t* esc_count_small;     // (zeroed) -- the small-tile AC-ESC's list, counter
   int64_t* esc_next_small;      // (zeroed)
+  int64_t* rows_next;           // adaptive: batch counter of the persistent k_rows (zeroed)
 };
 void launch_esc(const EscArgs& a, bool f64, cudaStream_t st);
-// adaptive strategy: lists of the blocks k_hash left (big / small tile), before the ESCs
-void launch_esc_lists(const EscArgs& a, cudaStream_t st);
 // adaptive alternative (hash.cu, reading R31): must run before launch_esc on the same stream
 void launch_hash(const EscArgs& a, bool f64, cudaStream_t st);
 // column-dictionary accumulator (dict.cu, reading R33): runs before launch_hash on the
 // same stream; blocks it finishes get hash_done = 2, the rest stay hash candidates
 void launch_dict(const EscArgs& a, bool f64, cudaStream_t st);
 // per-row accumulator for blocks of short rows (rows.cu, reading R34): after launch_hash,
-// on the blocks no accumulator finished; the ones it finishes get hash_done = 3
+// on the blocks no accumulator finished; the ones it finishes get hash_done = 3, the
+// others go onto the AC-ESC lists (esc_list / esc_list_small) for launch_esc
 void launch_rows(const EscArgs& a, bool f64, cudaStream_t st);
 
 // ---- stage 3: chunk ordering, shared rows, merges (merge.cu) --------------------
@@ -119,6 +128,7 @@ struct MergeLists {
   int64_t* scan_tmp;
 };
 // shared rows, their kinds and merge offsets in one pass (lists sized by m.max_chunks)
+// L.counts_dev[0 .. 6) must be zero on entry.
 void launch_find_shared(const MergeState& m, const MergeLists& L, int64_t* total_shared_dev, cudaStream_t st);
 void launch_multi_groups(const MergeLists& L, int64_t nmulti, int64_t ngroups, cudaStream_t st);
 
@@ -181,6 +191,9 @@ void launch_rowptr_out(int64_t* dst, const int64_t* src, int64_t n, int64_t off,
 void launch_copy_offset(int32_t* dst, const int32_t* src, int64_t n, int32_t off, cudaStream_t st);
 // nbytes (multiple of 4, <= 4096) from device memory to mapped host memory, by a kernel
 void launch_read_back(const void* src, void* mapped_dst, int nbytes, cudaStream_t st);
+// two read-backs in one launch
+void launch_read_back2(const void* src1, void* mapped_dst1, int nbytes1, const void* src2, void* mapped_dst2,
+                       int nbytes2, cudaStream_t st);
 // p[i] += off for i < n (row pointers of a row piece placed after earlier pieces)
 void launch_add_offset(int32_t* p, int64_t n, int32_t off, cudaStream_t st);
 

@@ -140,6 +140,23 @@ acspgemm_status ensure(DevBuf& b, size_t bytes) {
     if (s_ != ACSPGEMM_OK) return s_;                   \
   } while (0)
 
+// scan_tmp: zero when (re)allocated; the scans leave it zero (scan.cu)
+acspgemm_status ensure_scan_tmp(DevBuf& b, int64_t elems, cudaStream_t st) {
+  void* old = b.p;
+  acspgemm_status s = ensure(b, sizeof(int64_t) * elems);
+  if (s == ACSPGEMM_OK && b.p != old) {
+    cudaError_t e = cudaMemsetAsync(b.p, 0, b.bytes, st);
+    if (e != cudaSuccess) return set_err(ACSPGEMM_ERR_CUDA, std::string("cudaMemsetAsync: ") + cudaGetErrorString(e));
+  }
+  return s;
+}
+
+#define ACS_ENSURE_SCAN_TMP(buf, elems, st)                  \
+  do {                                                       \
+    acspgemm_status s_ = ensure_scan_tmp((buf), (elems), (st)); \
+    if (s_ != ACSPGEMM_OK) return s_;                        \
+  } while (0)
+
 template <typename P>
 P* ptr(DevBuf& b) { return reinterpret_cast<P*>(b.p); }
 
@@ -178,7 +195,9 @@ int64_t helper_bytes(acspgemm_plan p) {
 
 // Read n device words into h_scal (a host round trip), recorded for pattern replay; in
 // replay the recorded values are used instead (no launch, no synchronisation).
-acspgemm_status sync_read(acspgemm_plan p, const int64_t* dev, int n, cudaStream_t st) {
+// extra_*: a second read-back in the same launch (not recorded; skipped in replay).
+acspgemm_status sync_read(acspgemm_plan p, const int64_t* dev, int n, cudaStream_t st, const void* extra_src = nullptr,
+                          void* extra_dst = nullptr, int extra_bytes = 0) {
   if (p->replay) {
     if (p->rec_pos >= p->rec.size() || (int)p->rec[p->rec_pos].size() != n)
       return set_err(ACSPGEMM_ERR_INTERNAL, "pattern replay out of step");
@@ -186,14 +205,15 @@ acspgemm_status sync_read(acspgemm_plan p, const int64_t* dev, int n, cudaStream
     ++p->rec_pos;
     return ACSPGEMM_OK;
   }
-  launch_read_back(dev, p->h_scal, (int)sizeof(int64_t) * n, st);
+  if (extra_src)
+    launch_read_back2(dev, p->h_scal, (int)sizeof(int64_t) * n, extra_src, extra_dst, extra_bytes, st);
+  else
+    launch_read_back(dev, p->h_scal, (int)sizeof(int64_t) * n, st);
   tl_launches += 1;
   ACS_CUDA(cudaStreamSynchronize(st));
   p->rec.emplace_back(p->h_scal, p->h_scal + n);
   return ACSPGEMM_OK;
 }
-
-__global__ void k_put_i64(int64_t* dst, const int32_t* src) { *dst = *src; }
 
 acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const acspgemm_csr_in* B,
                               acspgemm_dtype dtype, cudaStream_t st, int64_t* nnz_c) {
@@ -239,9 +259,9 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->scal, sizeof(int64_t) * 32);
   ACS_ENSURE(p->err, sizeof(int32_t) * 4);
   int64_t* scal = ptr<int64_t>(p->scal);
-  ACS_CUDA(cudaMemsetAsync(p->err.p, 0, sizeof(int32_t) * 4, st));
 
   if (p->opt.validate_inputs && !p->replay) {
+    ACS_CUDA(cudaMemsetAsync(p->err.p, 0, sizeof(int32_t) * 4, st));
     launch_validate(Av, ptr<int32_t>(p->err), st);
     launch_validate(Bv, ptr<int32_t>(p->err), st);
     tl_launches += 2;
@@ -284,29 +304,36 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->esc_list, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->esc_list_small, sizeof(int32_t) * max_blocks);
   const int64_t tmp_n = scan_tmp_elems(std::max<int64_t>(max_blocks, A->rows) * 2 + 1024);
-  ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * tmp_n);
+  ACS_ENSURE_SCAN_TMP(p->scan_tmp, tmp_n, st);
+  ACS_ENSURE(p->row_count, sizeof(int32_t) * A->rows);
   int32_t* nblocks_dev = reinterpret_cast<int32_t*>(scal + 20);
-  launch_segments(Av, nseg, explicit_rows, ptr<int64_t>(p->seg), nblocks_dev, st);
+  // scal words: 0 products, 1 slots, 2 nblocks, 3 ncand / total chunks, 4 max block
+  // products / shared rows, 5 chunk elements, 6 hash blocks, 7 dict blocks, 8..14 merge
+  // class counts, 15 k_rows blocks, 16 nnz(C), 20 nblocks (int32), 24-25 dense slices,
+  // 26 k_rows batches, 28-31 AC-ESC lists.  The counters are zeroed by k_segments, the
+  // first kernel (with err), and k_glb zeroes the per-row counters: no memset launches.
+  ZeroList zero{};
+  zero.p[0] = scal + 3; zero.n[0] = 2;
+  zero.p[1] = scal + 6; zero.n[1] = 10;
+  zero.p[2] = scal + 26; zero.n[2] = 6;
+  zero.p[3] = reinterpret_cast<int64_t*>(p->err.p); zero.n[3] = 2;
+  launch_segments(Av, nseg, explicit_rows, ptr<int64_t>(p->seg), nblocks_dev, st, zero);
   tl_launches += 1;
-  launch_glb(Av, nseg, ptr<int64_t>(p->seg), ptr<int32_t>(p->brs), max_blocks, st);
+  launch_glb(Av, nseg, ptr<int64_t>(p->seg), ptr<int32_t>(p->brs), max_blocks, st, ptr<int32_t>(p->row_count));
   tl_launches += 1;
-  ACS_CUDA(cudaMemsetAsync(scal + 3, 0, 2 * sizeof(int64_t), st));   // hash candidates (R31), max block products
   launch_block_bounds(Av, Bv, nseg, ptr<int64_t>(p->seg), nblocks_dev, max_blocks, ptr<int32_t>(p->nzb),
                       ptr<int32_t>(p->nze), ptr<int64_t>(p->bprod), ptr<int64_t>(p->bslot),
-                      p->opt.strategy != ACSPGEMM_STRATEGY_ESC ? ptr<int32_t>(p->hdone) : nullptr, scal + 3, scal + 4, st);
+                      p->opt.strategy != ACSPGEMM_STRATEGY_ESC ? ptr<int32_t>(p->hdone) : nullptr, scal + 3, scal + 4,
+                      scal + 2, st);
   tl_launches += 1;
   launch_scan_i64(ptr<int64_t>(p->bprod), ptr<int64_t>(p->pool_off), max_blocks, scal + 0, ptr<int64_t>(p->scan_tmp), st);
   launch_scan_i64(ptr<int64_t>(p->bslot), ptr<int64_t>(p->desc_off), max_blocks, scal + 1, ptr<int64_t>(p->scan_tmp), st);
-  tl_launches += 6;
-  k_put_i64<<<1, 1, 0, st>>>(scal + 2, nblocks_dev);
-  tl_launches += 1;
+  tl_launches += 2;
   ACS_CUDA(cudaGetLastError());
   // segment boundaries (for info) ride along with the first read-back (replay: unchanged)
-  if (!p->replay) {
-    launch_read_back(p->seg.p, p->h_scal + H_SEG_INFO, (int)sizeof(int64_t) * (nseg + 1), st);
-    tl_launches += 1;
-  }
-  if ((s = sync_read(p, scal, 5, st)) != ACSPGEMM_OK) return s;
+  if ((s = sync_read(p, scal, 5, st, p->seg.p, p->h_scal + H_SEG_INFO, (int)sizeof(int64_t) * (nseg + 1))) !=
+      ACSPGEMM_OK)
+    return s;
   const int64_t products = p->h_scal[0], slots = p->h_scal[1], nblocks = p->h_scal[2], ncand = p->h_scal[3];
   if (p->h_scal[4] > 0)
     return set_err(ACSPGEMM_ERR_INDEX_OVERFLOW, "a block of NPB nonzeros of A has " + std::to_string(p->h_scal[4]) +
@@ -322,11 +349,9 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->pool_col, sizeof(int32_t) * products);
   ACS_ENSURE(p->pool_val, (size_t)vbytes * products);
   ACS_ENSURE(p->descs, sizeof(ChunkDesc) * slots);
-  ACS_ENSURE(p->row_count, sizeof(int32_t) * A->rows);
   // scans later run over up to `slots` chunks / shared rows
-  ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * scan_tmp_elems(std::max<int64_t>(std::max(max_blocks, A->rows), slots) + 1));
+  ACS_ENSURE_SCAN_TMP(p->scan_tmp, scan_tmp_elems(std::max<int64_t>(std::max(max_blocks, A->rows), slots) + 1), st);
   p->info.pool_bytes = (int64_t)(p->pool_col.bytes + p->pool_val.bytes);
-  ACS_CUDA(cudaMemsetAsync(p->row_count.p, 0, sizeof(int32_t) * A->rows, st));
 
   // ------------------------------------------------------------ ESC -----------
   record(p, S_ESC, st);
@@ -348,13 +373,11 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.hash_done = nullptr;
   ea.hash_count = scal + 6;
   ea.dict_count = scal + 7;
-  ea.rows_count = scal + 2;              // free after the first read-back
+  ea.rows_count = scal + 15;
   ea.esc_list = ptr<int32_t>(p->esc_list);
   ea.esc_count = scal + 28;
   ea.esc_next = scal + 29;
-  ACS_CUDA(cudaMemsetAsync(scal + 6, 0, 2 * sizeof(int64_t), st));
-  ACS_CUDA(cudaMemsetAsync(scal + 2, 0, sizeof(int64_t), st));
-  ACS_CUDA(cudaMemsetAsync(scal + 28, 0, 2 * sizeof(int64_t), st));
+  ea.rows_next = scal + 26;
   ea.blk_products = ptr<int64_t>(p->bprod);
   ea.esc_list_small = nullptr;
   ea.trace = nullptr;
@@ -371,7 +394,6 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   if (p->opt.strategy != ACSPGEMM_STRATEGY_ESC) {
     // hash accumulator first (reading R31); blocks it does not finish go to AC-ESC,
     // small ones (<= 512 products) to the small-tile AC-ESC (reading R32)
-    ACS_CUDA(cudaMemsetAsync(scal + 30, 0, 2 * sizeof(int64_t), st));
     ea.hash_done = ptr<int32_t>(p->hdone);
     ea.esc_list_small = ptr<int32_t>(p->esc_list_small);
   }
@@ -396,10 +418,9 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     tl_launches += nblocks > 0 ? 1 : 0;
   }
   if (ea.hash_done) {
-    launch_esc_lists(ea, st);
     ea.trace = trace_of(3);
-    acs_launch_esc_small(&ea, p->f64, st);
-    tl_launches += nblocks > 0 ? 2 : 0;
+    acs_launch_esc_small(&ea, p->f64, st);   // k_rows listed the blocks left to AC-ESC
+    tl_launches += nblocks > 0 ? 1 : 0;
   }
   ea.trace = trace_of(2);
   launch_esc(ea, p->f64, st);
@@ -415,7 +436,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->shared, sizeof(SharedRow) * slots);
   launch_scan_i32(ptr<int32_t>(p->nchunks), ptr<int64_t>(p->chunk_base), nblocks, scal + 3, ptr<int64_t>(p->scan_tmp), st);
   launch_scan_i32(ptr<int32_t>(p->bused), ptr<int64_t>(p->bused_scan), nblocks, scal + 5, ptr<int64_t>(p->scan_tmp), st);
-  tl_launches += 6;
+  tl_launches += 2;
   MergeState ms;
   ms.nblocks = (int32_t)nblocks;
   ms.desc_off = ptr<int64_t>(p->desc_off);
@@ -457,10 +478,10 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   L.scan_tmp = ptr<int64_t>(p->scan_tmp);
   launch_gather_chunks(ms, st);
   launch_find_shared(ms, L, scal + 4, st);
-  tl_launches += 1 + (slots > 0 ? 11 : 0);
+  tl_launches += 1 + (slots > 0 ? 7 : 0);
   ACS_CUDA(cudaGetLastError());
-  if ((s = sync_read(p, scal + 2, 12, st)) != ACSPGEMM_OK) return s;
-  p->info.nrow_blocks = p->h_scal[0];
+  if ((s = sync_read(p, scal + 2, 14, st)) != ACSPGEMM_OK) return s;
+  p->info.nrow_blocks = p->h_scal[13];
   p->info.nhash_blocks = p->h_scal[4];
   p->info.ndict_blocks = p->h_scal[5];
   p->total_chunks = p->h_scal[1];
@@ -491,7 +512,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
       ACS_ENSURE(p->gstart, sizeof(int32_t) * 2 * (gmax + 1));
       L.group_start = ptr<int32_t>(p->gstart);
       launch_multi_groups(L, nmulti, gmax, st);
-      tl_launches += 1 + 3 + 1 + 1;
+      tl_launches += 1 + 1 + 1 + 1;
       ngroups = gmax;
     }
     ACS_ENSURE(p->merge_col, sizeof(int32_t) * merge_total);
@@ -540,21 +561,21 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
       g.gbase = ptr<int64_t>(p->g_base);
       launch_giant_span(ma, g, st);
       launch_scan_i64(g.gnsl, g.gbase, ngiant, scal + 24, ptr<int64_t>(p->scan_tmp), st);
-      tl_launches += 1 + 3;
+      tl_launches += 1 + 1;
       ACS_CUDA(cudaGetLastError());
       if ((s = sync_read(p, scal + 24, 1, st)) != ACSPGEMM_OK) return s;
       const int64_t nslices = p->h_scal[0];
       ACS_ENSURE(p->g_tcol, sizeof(int32_t) * nslices);            // entries per slice
       ACS_ENSURE(p->g_tval, sizeof(int64_t) * nslices);            // their scan
       ACS_ENSURE(p->g_tcnt, sizeof(int32_t) * nslices);
-      ACS_ENSURE(p->scan_tmp, sizeof(int64_t) * scan_tmp_elems(nslices + 1));
+      ACS_ENSURE_SCAN_TMP(p->scan_tmp, scan_tmp_elems(nslices + 1), st);
       g.gent = ptr<int32_t>(p->g_tcol);
       g.gpos = ptr<int64_t>(p->g_tval);
       g.tcnt = ptr<int32_t>(p->g_tcnt);
       launch_giant_count(ma, g, nslices, st);
       launch_scan_i32(g.gent, g.gpos, nslices, scal + 25, ptr<int64_t>(p->scan_tmp), st);
       launch_giant_merge(ma, g, nslices, p->f64, st);
-      tl_launches += 1 + 3 + 2;
+      tl_launches += 1 + 1 + 2;
     }
     ACS_CUDA(cudaGetLastError());
   } else {
@@ -574,7 +595,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->row_ptr, sizeof(int64_t) * (A->rows + 1));
   launch_scan_rowptr(ptr<int32_t>(p->row_count), ptr<int64_t>(p->row_ptr), A->rows, scal + 16,
                      ptr<int64_t>(p->scan_tmp), st);
-  tl_launches += 3;
+  tl_launches += 1;
   ACS_CUDA(cudaGetLastError());
   record(p, S_CC, st);
   int64_t nnz;
@@ -586,9 +607,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     errflag = (int32_t)p->rec[p->rec_pos][1];
     ++p->rec_pos;
   } else {
-    launch_read_back(scal + 16, p->h_scal, sizeof(int64_t), st);
-    launch_read_back(p->err.p, p->h_scal + 1, sizeof(int32_t), st);
-    tl_launches += 2;
+    launch_read_back2(scal + 16, p->h_scal, sizeof(int64_t), p->err.p, p->h_scal + 1, sizeof(int32_t), st);
+    tl_launches += 1;
     ACS_CUDA(cudaStreamSynchronize(st));
     nnz = p->h_scal[0];
     errflag = *reinterpret_cast<int32_t*>(p->h_scal + 1);

@@ -53,16 +53,23 @@ struct RowsSmem {
   int wout[ROWS_WARPS][5];
   alignas(8) int scratch[40];
   int flag;
+  int batch[32];                 // the current batch's blocks no accumulator finished
+  int nbatch, bbase;
 };
 
+// A block left to AC-ESC: onto the big- or small-tile list (reading R32).
+__device__ __forceinline__ void rows_give_up(const EscArgs& a, int b) {
+  const bool small = a.esc_list_small && a.blk_products[b] <= CAP_SMALL;
+  int64_t* cnt = small ? a.esc_count_small : a.esc_count;
+  int32_t* list = small ? a.esc_list_small : a.esc_list;
+  list[atomicAdd(reinterpret_cast<unsigned long long*>(cnt), 1ull)] = b;
+}
+
+// One block: finished here (hash_done[b] = 3) or left to AC-ESC (listed).
 template <typename T>
-__global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  RowsSmem<T>& S = *reinterpret_cast<RowsSmem<T>*>(smem_raw);
+__device__ __forceinline__ void rows_block(RowsSmem<T>& S, const EscArgs& a, const int b) {
   const unsigned FULL = 0xffffffffu;
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-  const int b = blockIdx.x;
-  if (a.hash_done[b] != 0) return;       // finished by an accumulator already
   const uint64_t t_start = a.trace ? global_timer() : 0;
   const int32_t* __restrict__ bcol = a.B.col;
   const T* __restrict__ bval = reinterpret_cast<const T*>(a.B.val);
@@ -72,7 +79,10 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
                                 nent, total);
   bool big = false;
   for (int r = tid; r < nrows; r += THREADS) big |= S.wd[S.row_first[r + 1]] - S.wd[S.row_first[r]] > ROWS_PMAX;
-  if (__syncthreads_or(big)) return;     // a long row: AC-ESC
+  if (__syncthreads_or(big)) {           // a long row: AC-ESC
+    if (tid == 0) rows_give_up(a, b);
+    return;
+  }
   split_rows<ROWS_WARPS>(S.wd, S.row_first, nrows, total, S.wrow);
   __syncthreads();
   const int rlo = S.wrow[w], rhi = S.wrow[w + 1];
@@ -179,9 +189,47 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
   }
   __syncthreads();
   if (tid == 0) trace_block(a.trace, b, t_start);
-  if (tid == 0 && !S.flag) {
-    emit_warp_chunks(a, b, ROWS_WARPS, S.wrow, S.wout, S.wd, S.row_first, a.rows_count);
-    a.hash_done[b] = 3;
+  if (tid == 0) {
+    if (!S.flag) {
+      emit_warp_chunks(a, b, ROWS_WARPS, S.wrow, S.wout, S.wd, S.row_first, a.rows_count);
+      a.hash_done[b] = 3;
+    } else {
+      rows_give_up(a, b);
+    }
+  }
+}
+
+// Persistent: a CTA takes ROWS_BATCH consecutive block numbers at a time (rows_next),
+// keeps those no accumulator finished (hash_done == 0, in order) and runs them; the blocks
+// it gives up go onto the AC-ESC lists, so there is no list pass and no grid of nblocks
+// CTAs that mostly exit at once (cfg2: all 108,880 blocks are k_hash's).
+constexpr int ROWS_BATCH = 32;
+
+template <typename T>
+__global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  RowsSmem<T>& S = *reinterpret_cast<RowsSmem<T>*>(smem_raw);
+  const int tid = threadIdx.x;
+  for (;;) {
+    if (tid < 32) {
+      int base = 0;
+      if (tid == 0)
+        base = (int)atomicAdd(reinterpret_cast<unsigned long long*>(a.rows_next), (unsigned long long)ROWS_BATCH);
+      base = __shfl_sync(0xffffffffu, base, 0);
+      const int b = base + tid;
+      const bool need = b < a.nblocks && a.hash_done[b] == 0;
+      const unsigned m = __ballot_sync(0xffffffffu, need);
+      if (need) S.batch[__popc(m & ((1u << tid) - 1u))] = b;
+      if (tid == 0) { S.nbatch = __popc(m); S.bbase = base; }
+    }
+    __syncthreads();
+    const int bbase = S.bbase, n = S.nbatch;
+    __syncthreads();                     // read before warp 0 overwrites them (n == 0)
+    if (bbase >= a.nblocks) break;
+    for (int k = 0; k < n; ++k) {
+      rows_block<T>(S, a, S.batch[k]);
+      __syncthreads();                   // shared memory is reused by the next block
+    }
   }
 }
 
@@ -189,7 +237,13 @@ template <typename T>
 static void launch_rows_t(const EscArgs& a, cudaStream_t st) {
   const size_t smem = sizeof(RowsSmem<T>);
   cudaFuncSetAttribute(k_rows<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k_rows<T><<<a.nblocks, THREADS, smem, st>>>(a);
+  int dev = 0, sms = 148, per = 1;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_rows<T>, THREADS, smem);
+  const int64_t batches = (a.nblocks + ROWS_BATCH - 1) / ROWS_BATCH;
+  const int grid = (int)std::min<int64_t>(batches, (int64_t)sms * std::max(per, 1));
+  k_rows<T><<<grid, THREADS, smem, st>>>(a);
 }
 
 void launch_rows(const EscArgs& a, bool f64, cudaStream_t st) {
