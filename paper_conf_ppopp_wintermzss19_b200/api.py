@@ -162,9 +162,17 @@ class Plan:
             raise AcspgemmError(3, "Plan.multiply: nnz(C) >= 2^31 needs index64=True")   # INDEX_OVERFLOW
         dev = A.val.device
         rows = self._rows
-        rp = torch.empty(rows + 1, dtype=torch.int64 if index64 else torch.int32, device=dev)
-        col = torch.empty(max(nnz, 1), dtype=torch.int32, device=dev)
-        val = torch.empty(max(nnz, 1), dtype=A.dtype, device=dev)
+        # one allocation for C (row_ptr | col | val, each 256-byte aligned): the host gap
+        # between the symbolic read-back and the numeric launches is on the critical path
+        rdt = torch.int64 if index64 else torch.int32
+        rpb = (rows + 1) * (8 if index64 else 4)
+        n1 = max(nnz, 1)
+        o1 = (rpb + 255) // 256 * 256
+        o2 = o1 + (n1 * 4 + 255) // 256 * 256
+        buf = torch.empty(o2 + n1 * A.val.element_size(), dtype=torch.uint8, device=dev)
+        rp = buf[:rpb].view(rdt)
+        col = buf[o1:o1 + n1 * 4].view(torch.int32)
+        val = buf[o2:].view(A.dtype)
         self.numeric(rp, col, val, stream)
         return DeviceCSR(rows, B.cols, rp, col[:nnz], val[:nnz])
 

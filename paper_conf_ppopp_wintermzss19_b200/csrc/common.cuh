@@ -47,7 +47,10 @@ constexpr int PATH_MAX_CHUNKS = 32;          // Path Merge limit (reading R12)
 constexpr int PTR_LEN = ACS_PTR_LEN;
 constexpr int PTR_MAX = 160;
 constexpr int SEARCH_MAXP = 1024;            // Search Merge limit; longer chunk lists: dense slices (R30)
-constexpr int GIANT_SLICE = 4096;            // columns per dense-slice CTA
+#ifndef ACS_GIANT_SLICE
+#define ACS_GIANT_SLICE 8192
+#endif
+constexpr int GIANT_SLICE = ACS_GIANT_SLICE;  // columns of a dense slice (one accumulator)
 #ifndef ACS_DENSE_SPAN_RATIO
 #define ACS_DENSE_SPAN_RATIO 16
 #endif

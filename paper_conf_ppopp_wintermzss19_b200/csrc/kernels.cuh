@@ -157,8 +157,12 @@ struct GiantArgs {                // dense-slice merge of rows with > SEARCH_MAX
   const int32_t* list;            // [n] indices into shared
   int64_t n;
   int32_t* glo;                   // [n] first column of the row's span
+  int32_t* ghi;                   // [n] last column of the row's span
   int64_t* gnsl;                  // [n] slices of the row
   int64_t* gbase;                 // [n] exclusive scan of gnsl
+  int64_t* gmn;                   // [n] slices x pieces of the row
+  int64_t* gmbase;                // [n] exclusive scan of gmn
+  int32_t* pos;                   // [sum gmn] start of each piece's entries in each slice
   int32_t* gent;                  // [nslices] pre-merge entries per slice
   int64_t* gpos;                  // [nslices] exclusive scan of gent
   int32_t* tcnt;                  // [nslices] merged entries per slice

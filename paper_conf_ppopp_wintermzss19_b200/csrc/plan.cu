@@ -77,7 +77,7 @@ struct acspgemm_plan_s {
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan, hdone, esc_list, esc_list_small;
-  DevBuf lgiant, g_lo, g_nsl, g_base, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30): lists, spans, slices
+  DevBuf lgiant, g_lo, g_nsl, g_base, g_pos, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30): lists, spans, slices
   DevBuf trace;                  // acspgemm_set_trace: per block (SM, start, end) x 4 kernels (mpL)
   bool trace_on = false;
   int64_t trace_blocks = 0;
@@ -550,32 +550,38 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     if (nsearch > 0) { launch_search_merge(ma, p->f64, st); tl_launches += 1; }
     if (ngiant > 0) {
       // rows of > SEARCH_MAXP chunks: dense column slices (reading R30)
-      ACS_ENSURE(p->g_lo, sizeof(int32_t) * ngiant);
-      ACS_ENSURE(p->g_nsl, sizeof(int64_t) * ngiant);
-      ACS_ENSURE(p->g_base, sizeof(int64_t) * ngiant);
+      ACS_ENSURE(p->g_lo, sizeof(int32_t) * 2 * ngiant);          // first | last column
+      ACS_ENSURE(p->g_nsl, sizeof(int64_t) * 2 * ngiant);         // slices | slices x pieces
+      ACS_ENSURE(p->g_base, sizeof(int64_t) * 2 * ngiant);        // their scans
       GiantArgs g;
       g.list = ptr<int32_t>(p->lgiant);
       g.n = ngiant;
       g.glo = ptr<int32_t>(p->g_lo);
+      g.ghi = g.glo + ngiant;
       g.gnsl = ptr<int64_t>(p->g_nsl);
+      g.gmn = g.gnsl + ngiant;
       g.gbase = ptr<int64_t>(p->g_base);
+      g.gmbase = g.gbase + ngiant;
       launch_giant_span(ma, g, st);
+      launch_scan_i64(g.gmn, g.gmbase, ngiant, scal + 23, ptr<int64_t>(p->scan_tmp), st);
       launch_scan_i64(g.gnsl, g.gbase, ngiant, scal + 24, ptr<int64_t>(p->scan_tmp), st);
-      tl_launches += 1 + 1;
+      tl_launches += 1 + 2;
       ACS_CUDA(cudaGetLastError());
-      if ((s = sync_read(p, scal + 24, 1, st)) != ACSPGEMM_OK) return s;
-      const int64_t nslices = p->h_scal[0];
+      if ((s = sync_read(p, scal + 23, 2, st)) != ACSPGEMM_OK) return s;
+      const int64_t npos = p->h_scal[0], nslices = p->h_scal[1];
+      ACS_ENSURE(p->g_pos, sizeof(int32_t) * npos);
       ACS_ENSURE(p->g_tcol, sizeof(int32_t) * nslices);            // entries per slice
       ACS_ENSURE(p->g_tval, sizeof(int64_t) * nslices);            // their scan
       ACS_ENSURE(p->g_tcnt, sizeof(int32_t) * nslices);
       ACS_ENSURE_SCAN_TMP(p->scan_tmp, scan_tmp_elems(nslices + 1), st);
+      g.pos = ptr<int32_t>(p->g_pos);
       g.gent = ptr<int32_t>(p->g_tcol);
       g.gpos = ptr<int64_t>(p->g_tval);
       g.tcnt = ptr<int32_t>(p->g_tcnt);
       launch_giant_count(ma, g, nslices, st);
       launch_scan_i32(g.gent, g.gpos, nslices, scal + 25, ptr<int64_t>(p->scan_tmp), st);
       launch_giant_merge(ma, g, nslices, p->f64, st);
-      tl_launches += 1 + 1 + 2;
+      tl_launches += 2 + 1 + 2;
     }
     ACS_CUDA(cudaGetLastError());
   } else {
@@ -816,7 +822,7 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
                   &p->scan_tmp, &p->kflag, &p->kpos, &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan,
                   &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
                   &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->lgiant, &p->g_lo, &p->g_nsl,
-                  &p->g_base, &p->g_tcol, &p->g_tval, &p->g_tcnt, &p->hdone, &p->esc_list,
+                  &p->g_base, &p->g_pos, &p->g_tcol, &p->g_tval, &p->g_tcnt, &p->hdone, &p->esc_list,
                   &p->esc_list_small, &p->trace};
   for (DevBuf* b : bs) free_buf(*b);
   for (auto& pb : p->bp) for (DevBuf& b : pb) free_buf(b);
