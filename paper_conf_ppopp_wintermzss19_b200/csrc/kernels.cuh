@@ -80,6 +80,7 @@ struct EscArgs {
   int64_t* esc_count_small;     // (zeroed) -- the small-tile AC-ESC's list, counter
   int64_t* esc_next_small;      // (zeroed)
   int64_t* rows_next;           // adaptive: batch counter of the persistent k_rows (zeroed)
+  int32_t rows_batch;           // blocks per k_rows batch, 0: one CTA per block (set by launch_rows)
 };
 void launch_esc(const EscArgs& a, bool f64, cudaStream_t st);
 // adaptive alternative (hash.cu, reading R31): must run before launch_esc on the same stream
@@ -90,7 +91,8 @@ void launch_dict(const EscArgs& a, bool f64, cudaStream_t st);
 // per-row accumulator for blocks of short rows (rows.cu, reading R34): after launch_hash,
 // on the blocks no accumulator finished; the ones it finishes get hash_done = 3, the
 // others go onto the AC-ESC lists (esc_list / esc_list_small) for launch_esc
-void launch_rows(const EscArgs& a, bool f64, cudaStream_t st);
+// hash_ran: an accumulator ran before (persistent batches), else one CTA per block
+void launch_rows(const EscArgs& a, bool f64, bool hash_ran, cudaStream_t st);
 
 // ---- stage 3: chunk ordering, shared rows, merges (merge.cu) --------------------
 struct MergeState {

@@ -414,7 +414,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   record(p, S_HASHEND, st);
   if (ea.hash_done) {
     ea.trace = trace_of(1);
-    launch_rows(ea, p->f64, st);         // blocks of short rows (reading R34)
+    launch_rows(ea, p->f64, ncand > 0, st);   // blocks of short rows (reading R34)
     tl_launches += nblocks > 0 ? 1 : 0;
   }
   if (ea.hash_done) {

@@ -199,10 +199,11 @@ __device__ __forceinline__ void rows_block(RowsSmem<T>& S, const EscArgs& a, con
   }
 }
 
-// Persistent: a CTA takes ROWS_BATCH consecutive block numbers at a time (rows_next),
-// keeps those no accumulator finished (hash_done == 0, in order) and runs them; the blocks
-// it gives up go onto the AC-ESC lists, so there is no list pass and no grid of nblocks
-// CTAs that mostly exit at once (cfg2: all 108,880 blocks are k_hash's).
+// The blocks it gives up go onto the AC-ESC lists (no list pass).  Without a hash
+// candidate it runs one CTA per block; after k_hash / k_dict (most blocks done) it is
+// persistent: a CTA takes rows_batch (<= ROWS_BATCH) consecutive block numbers at a time
+// (rows_next) and runs those no accumulator finished (hash_done == 0, in order) -- no
+// grid of nblocks CTAs that mostly exit at once (cfg2: all 108,880 blocks are k_hash's).
 constexpr int ROWS_BATCH = 32;
 
 template <typename T>
@@ -210,14 +211,18 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   RowsSmem<T>& S = *reinterpret_cast<RowsSmem<T>*>(smem_raw);
   const int tid = threadIdx.x;
+  if (a.rows_batch == 0) {               // one CTA per block (most blocks are k_rows' own)
+    if (a.hash_done[blockIdx.x] == 0) rows_block<T>(S, a, blockIdx.x);
+    return;
+  }
   for (;;) {
     if (tid < 32) {
       int base = 0;
       if (tid == 0)
-        base = (int)atomicAdd(reinterpret_cast<unsigned long long*>(a.rows_next), (unsigned long long)ROWS_BATCH);
+        base = (int)atomicAdd(reinterpret_cast<unsigned long long*>(a.rows_next), (unsigned long long)a.rows_batch);
       base = __shfl_sync(0xffffffffu, base, 0);
       const int b = base + tid;
-      const bool need = b < a.nblocks && a.hash_done[b] == 0;
+      const bool need = tid < a.rows_batch && b < a.nblocks && a.hash_done[b] == 0;
       const unsigned m = __ballot_sync(0xffffffffu, need);
       if (need) S.batch[__popc(m & ((1u << tid) - 1u))] = b;
       if (tid == 0) { S.nbatch = __popc(m); S.bbase = base; }
@@ -234,21 +239,31 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
 }
 
 template <typename T>
-static void launch_rows_t(const EscArgs& a, cudaStream_t st) {
+static void launch_rows_t(const EscArgs& a, bool hash_ran, cudaStream_t st) {
   const size_t smem = sizeof(RowsSmem<T>);
   cudaFuncSetAttribute(k_rows<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int dev = 0, sms = 148, per = 1;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_rows<T>, THREADS, smem);
-  const int64_t batches = (a.nblocks + ROWS_BATCH - 1) / ROWS_BATCH;
-  const int grid = (int)std::min<int64_t>(batches, (int64_t)sms * std::max(per, 1));
-  k_rows<T><<<grid, THREADS, smem, st>>>(a);
+  // batches of up to ROWS_BATCH blocks, at least ~16 per CTA (a short tail), one block
+  // per batch when there are fewer blocks than CTAs
+  const int64_t slots = (int64_t)sms * std::max(per, 1);
+  EscArgs b = a;
+  if (!hash_ran) {                       // no accumulator ran: one CTA per block
+    b.rows_batch = 0;
+    k_rows<T><<<a.nblocks, THREADS, smem, st>>>(b);
+    return;
+  }
+  b.rows_batch = (int)std::max<int64_t>(1, std::min<int64_t>(ROWS_BATCH, a.nblocks / (slots * 16)));
+  const int64_t batches = (a.nblocks + b.rows_batch - 1) / b.rows_batch;
+  const int grid = (int)std::min<int64_t>(batches, slots);
+  k_rows<T><<<grid, THREADS, smem, st>>>(b);
 }
 
-void launch_rows(const EscArgs& a, bool f64, cudaStream_t st) {
+void launch_rows(const EscArgs& a, bool f64, bool hash_ran, cudaStream_t st) {
   if (a.nblocks <= 0) return;
-  if (f64) launch_rows_t<double>(a, st); else launch_rows_t<float>(a, st);
+  if (f64) launch_rows_t<double>(a, hash_ran, st); else launch_rows_t<float>(a, hash_ran, st);
 }
 
 }  // namespace acs
