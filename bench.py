@@ -291,15 +291,30 @@ def kernel_roofline(cfg, dtype, st_list, info, rows_a, nnz_a, rows_b, nnz_b, vby
         byts += info["products"] * e
     achieved = byts / (ms * 1e-3) / 1e9
     traffic = None
+    issue = None
     tf = os.path.join(ROOT, "profiles", f"{tag}_traffic_{cfg}_{dtype}.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get("dram_bytes_per_launch")
+            prof = json.load(open(tf))
+            traffic = prof.get("dram_bytes_per_launch")
+            inst = prof.get("metrics", {}).get("smsp__inst_executed.sum")
+            if inst:
+                # the issue-rate ceiling the counters show this kernel is near: warp
+                # instructions per launch (committed ncu capture) over the live launch
+                # time, against 4 schedulers x SMs x the max SM clock (one warp
+                # instruction per scheduler per cycle)
+                import torch
+                sms = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+                mhz = float(os.environ.get("ACS_SM_MAX_MHZ", "1965"))
+                ipk = inst / (ms * 1e-3) / 1e9
+                pk = 4 * sms * mhz * 1e-3
+                issue = {"achieved": ipk, "peak": pk, "unit": "G warp-instr/s", "frac": ipk / pk,
+                         "warp_instr_per_launch": inst, "peak_source": f"4 x {sms} SMs x {mhz:.0f} MHz"}
         except Exception:
             traffic = None
     return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
             "traffic": traffic, "kernel": kern, "algorithmic_bytes_per_launch": byts, "avg_launch_ms": ms,
-            "peak_source": peak_src}
+            "peak_source": peak_src, "issue": issue}
 
 
 def segment_digest(torch, C, seg_rows_local):

@@ -258,3 +258,25 @@ def test_sm_load_trace(cuda_available):
     with pytest.raises(p.AcspgemmError):
         plan.sm_load("esc")
     plan.close()
+
+
+def test_plan_reuse_scan_state_many_tiles(cuda_available):
+    """The one-pass scans keep a ticket, a done counter and per-tile posts in plan memory
+    and leave them zero (scan.cu).  Alternate large (many tiles: 70,001 rows = 69 tiles
+    of the row-pointer scan) and tiny multiplies on one plan, and a multiply with a
+    capture in between (numeric_update), and check every C exactly."""
+    p = pkg()
+    plan = p.Plan()
+    big = random_csr(70001, 70001, 4e-5, seed=31)
+    mid = power_law_csr(9000, 9000, 6, 1.4, 3000, seed=32)
+    tiny = poisson2d_5pt(3)
+    for A in (big, tiny, mid, big, tiny, big):
+        dA = dev(A)
+        C = plan.multiply(dA, dA)
+        check(C, A, A)
+        if A is mid:
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                plan.numeric_update(dA, dA, C, s)
+            s.synchronize()
+            check(C, A, A)
