@@ -46,7 +46,7 @@
 extern "C" {
 #endif
 
-#define ACSPGEMM_ABI_VERSION 1
+#define ACSPGEMM_ABI_VERSION 2   /* 2: acspgemm_options.pool_mode, acspgemm_info.pool_mode / ndeferred_blocks */
 
 typedef enum { ACSPGEMM_F32 = 0, ACSPGEMM_F64 = 1 } acspgemm_dtype;
 
@@ -89,7 +89,7 @@ typedef struct acspgemm_plan_s* acspgemm_plan;
 
 typedef struct {
   size_t pool_limit_bytes;   /* 0 = no limit; else symbolic fails with OUT_OF_MEMORY when the
-                                exact chunk-pool bound (products x (4 + value size)) exceeds it */
+                                chunk pool the pool_mode sizes exceeds it */
   int validate_inputs;       /* 1: check that A and B are canonical CSR (one extra sync) */
   int collect_stage_times;   /* 1: record CUDA events between stages (acspgemm_stage_times) */
   int num_segments;          /* canonical segments S (default 8, max 64) */
@@ -100,7 +100,22 @@ typedef struct {
                                 ACSPGEMM_STRATEGY_HASH: hash accumulator, then AC-ESC;
                                 ACSPGEMM_STRATEGY_DICT: block dictionary (R33), hash, AC-ESC.
                                 ADAPTIVE, HASH and DICT give the same results bit for bit. */
+  int pool_mode;             /* chunk-pool sizing (L556, L580; reading R40):
+                                ACSPGEMM_POOL_EXACT (default): every block owns its exact product
+                                bound, products x (4 + value size) in all -- no overflow path;
+                                ACSPGEMM_POOL_BOUND: a hash-accumulator candidate block owns
+                                min(products, rows x 256) (the accumulators' output bound); a
+                                candidate that ends in AC-ESC is deferred and run after the first
+                                pass in a region of its exact bound appended to the pool (one more
+                                read-back; the pool grows by a copy).  Same bytes of C;
+                                ACSPGEMM_POOL_AUTO: EXACT when the exact bound fits
+                                pool_limit_bytes (or there is no limit), else BOUND.
+                                The DICT strategy always uses EXACT. */
 } acspgemm_options;
+
+#define ACSPGEMM_POOL_EXACT 0
+#define ACSPGEMM_POOL_BOUND 1
+#define ACSPGEMM_POOL_AUTO 2
 
 #define ACSPGEMM_STRATEGY_ADAPTIVE 0
 #define ACSPGEMM_STRATEGY_ESC 1
@@ -126,9 +141,12 @@ typedef struct {
   int64_t nhash_blocks;      /* blocks completed by an accumulator (dictionary or hash; R33, R31) */
   int64_t ndict_blocks;      /* of them, blocks completed by the column-dictionary accumulator (R33) */
   int64_t nrow_blocks;       /* blocks completed by the per-row accumulator for short rows (R34) */
+  int64_t ndeferred_blocks;  /* POOL_BOUND: candidate blocks that ended in AC-ESC (second pass) */
+  int32_t pool_mode;         /* the sizing the last symbolic used (EXACT or BOUND) */
 } acspgemm_info;
 
-/* Defaults: no pool limit, no validation, no stage times, 8 segments, adaptive strategy. */
+/* Defaults: no pool limit, no validation, no stage times, 8 segments, adaptive strategy,
+   exact pool. */
 void acspgemm_options_default(acspgemm_options* opt);
 
 /* Create a plan.  opt may be NULL (defaults).  *plan receives the handle. */

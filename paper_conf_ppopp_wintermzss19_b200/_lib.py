@@ -35,7 +35,7 @@ CsrOut64 = CsrOut
 class Options(ctypes.Structure):
     _fields_ = [("pool_limit_bytes", ctypes.c_size_t), ("validate_inputs", ctypes.c_int),
                 ("collect_stage_times", ctypes.c_int), ("num_segments", ctypes.c_int),
-                ("strategy", ctypes.c_int)]
+                ("strategy", ctypes.c_int), ("pool_mode", ctypes.c_int)]
 
 
 class Info(ctypes.Structure):
@@ -44,7 +44,8 @@ class Info(ctypes.Structure):
                 ("nsearch", I64), ("nmulti_groups", I64), ("merge_elems", I64),
                 ("pool_bytes", I64), ("helper_bytes", I64), ("pool_estimate_bytes", ctypes.c_double),
                 ("kernel_launches", I64), ("nsegments", I32), ("segment_rows", I64 * 65),
-                ("nhash_blocks", I64), ("ndict_blocks", I64), ("nrow_blocks", I64)]
+                ("nhash_blocks", I64), ("ndict_blocks", I64), ("nrow_blocks", I64),
+                ("ndeferred_blocks", I64), ("pool_mode", I32)]
 
 
 # name -> (restype, argtypes); every symbol include/acspgemm.h declares

@@ -84,19 +84,26 @@ def _stream_ptr(stream: Optional[torch.cuda.Stream]) -> ctypes.c_void_p:
 
 
 _STRATEGIES = {"adaptive": 0, "esc": 1, "hash": 2, "dict": 3}   # ACSPGEMM_STRATEGY_* (include/acspgemm.h)
+_POOL_MODES = {"exact": 0, "bound": 1, "auto": 2}               # ACSPGEMM_POOL_*
 
 
 class Plan:
     """A reusable multiply plan (owns the chunk pool and helper memory)."""
 
     def __init__(self, pool_limit_bytes: int = 0, validate: bool = False, stage_times: bool = False,
-                 num_segments: int = 8, strategy: str = "adaptive"):
+                 num_segments: int = 8, strategy: str = "adaptive", pool_mode: str = "exact"):
         """strategy: "adaptive" (hash accumulator per candidate block, per-row accumulator
         for blocks of short rows, AC-ESC fallback; readings R31, R34), "hash" (the same path;
         kept for the round-1 API), "dict" (column dictionary first, reading R33) -- these three give the
-        same bits -- or "esc" (every block through AC-ESC)."""
+        same bits -- or "esc" (every block through AC-ESC).
+        pool_mode: "exact" (every block its exact product bound), "bound" (accumulator
+        candidates bounded by rows x 256, their AC-ESC fallbacks deferred to a second
+        pass), "auto" (exact if it fits pool_limit_bytes, else bound) -- same bytes of C
+        (include/acspgemm.h, reading R40)."""
         if strategy not in _STRATEGIES:
             raise ValueError("strategy must be one of " + ", ".join(_STRATEGIES))
+        if pool_mode not in _POOL_MODES:
+            raise ValueError("pool_mode must be one of " + ", ".join(_POOL_MODES))
         lib = load()
         opt = Options()
         lib.acspgemm_options_default(ctypes.byref(opt))
@@ -105,6 +112,7 @@ class Plan:
         opt.collect_stage_times = int(bool(stage_times))
         opt.num_segments = int(num_segments)
         opt.strategy = _STRATEGIES[strategy]
+        opt.pool_mode = _POOL_MODES[pool_mode]
         h = ctypes.c_void_p()
         check(lib.acspgemm_plan_create(ctypes.byref(h), ctypes.byref(opt)), "acspgemm_plan_create")
         self._h = h

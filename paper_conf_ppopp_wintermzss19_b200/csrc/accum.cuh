@@ -190,15 +190,30 @@ __device__ __forceinline__ void split_rows(const int* wd, const int* row_first, 
 // One chunk descriptor per warp that emitted rows (L424-L428), in warp order = row
 // order; wout[q] = {count, first_row, last_row, first_count, last_count}; counts the
 // block in *counter (info only).  Thread 0.
-__device__ __forceinline__ void emit_warp_chunks(const EscArgs& a, int b, int nw, const int* wrow, const int (*wout)[5],
+// Where (relative to the block's pool region) the warp owning rows [rlo, ..) writes: exact
+// pools: after the products of the rows before it; POOL_BOUND (reading R40): after
+// sum min(products, HASH_UMAX) over them -- the accumulators' output bound, so the runs
+// pack into min(products, rows x HASH_UMAX).  All lanes of the warp call it.
+__device__ __forceinline__ int warp_out_base(const EscArgs& a, const int* wd, const int* row_first, int rlo,
+                                             int nrows, int lane) {
+  if (rlo >= nrows) return 0;
+  if (!a.bound) return wd[row_first[rlo]];
+  int s = 0;
+  for (int r = lane; r < rlo; r += 32) s += min(wd[row_first[r + 1]] - wd[row_first[r]], HASH_UMAX);
+  return __reduce_add_sync(0xffffffffu, s);
+}
+
+// wout[w]: count, first_row, last_row, first_count, last_count, warp_out_base
+__device__ __forceinline__ void emit_warp_chunks(const EscArgs& a, int b, int nw, const int* wrow, const int (*wout)[6],
                                                  const int* wd, const int* row_first, int64_t* counter) {
   const int64_t pool_base = a.pool_off[b];
   const int64_t desc_base = a.desc_off[b];
   int seq = 0, used = 0;
+  (void)wrow; (void)wd; (void)row_first;
   for (int q = 0; q < nw; ++q) {
     if (wout[q][0] == 0) continue;
     ChunkDesc d;
-    d.data_off = pool_base + wd[row_first[wrow[q]]];
+    d.data_off = pool_base + wout[q][5];
     d.first_row = wout[q][1];
     d.last_row = wout[q][2];
     d.count = wout[q][0];

@@ -98,7 +98,7 @@ struct DictSmem {
     DictWarp<T> w[DICT_WARPS];
   } u;
   int wrow[DICT_WARPS + 1];
-  int wout[DICT_WARPS][5];
+  int wout[DICT_WARPS][6];
   alignas(8) int scratch[40];
   int nd, cmin, cmax, bad;
 };
@@ -439,7 +439,8 @@ __global__ void __launch_bounds__(DICT_THREADS, DICT_WARPS == 8 ? 2 : 3) k_dict(
   for (int i = lane; i < DICT_DMAX + 32; i += 32) Wp.mark[i] = 0;
   __syncwarp();
   const int rlo = S.wrow[w], rhi = S.wrow[w + 1];
-  const int64_t wbase_pool = a.pool_off[b] + (rlo < nrows ? S.wd[S.row_first[rlo]] : 0);
+  const int wrel = warp_out_base(a, S.wd, S.row_first, rlo, nrows, lane);
+  const int64_t wbase_pool = a.pool_off[b] + wrel;
   T* pval = reinterpret_cast<T*>(a.pool_val);
   int32_t* pcol = a.pool_col;
   const int nwin = (D + 31) >> 5;
@@ -498,6 +499,7 @@ __global__ void __launch_bounds__(DICT_THREADS, DICT_WARPS == 8 ? 2 : 3) k_dict(
     S.wout[w][2] = last_row;
     S.wout[w][3] = first_count;
     S.wout[w][4] = last_count;
+    S.wout[w][5] = wrel;
   }
   __syncthreads();
   if (tid == 0) {

@@ -117,7 +117,8 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
                                int64_t max_blocks, int32_t* __restrict__ nz_begin, int32_t* __restrict__ nz_end,
                                int64_t* __restrict__ products, int64_t* __restrict__ slots,
                                int32_t* __restrict__ hash_ok, int64_t* __restrict__ ncand,
-                               int64_t* __restrict__ max_products, int64_t* __restrict__ nblocks_out) {
+                               int64_t* __restrict__ max_products, int64_t* __restrict__ nblocks_out,
+                               const int32_t* __restrict__ brs, int64_t rows_a, int64_t* __restrict__ est) {
   __shared__ int64_t s_nz[SEG_STRIDE], s_base[SEG_STRIDE];
   __shared__ int s_cand;
   for (int i = threadIdx.x; i <= nseg; i += blockDim.x) {
@@ -132,6 +133,7 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
   if (nblocks_out && blockIdx.x == 0 && threadIdx.x == 0) *nblocks_out = nblocks;
   if (b < max_blocks && b >= nblocks && lane == 0) {
     products[b] = 0; slots[b] = 0; nz_begin[b] = 0; nz_end[b] = 0;
+    if (est) est[b] = 0;
     if (hash_ok) hash_ok[b] = 0;
   }
   if (b < nblocks) {
@@ -205,6 +207,13 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
       if (hash_ok) hash_ok[b] = hok;
       if (hok) atomicAdd(&s_cand, 1);
       products[b] = sum;
+      if (est) {
+        // POOL_BOUND (reading R40): a candidate's accumulator output is at most HASH_UMAX
+        // columns per row (k_hash) or fewer (k_rows); its rows lie in [brs[b], brs[b+1]]
+        const int64_t last = b + 1 < nblocks ? (int64_t)brs[b + 1] : rows_a - 1;
+        const int64_t nr = last - brs[b] + 1;
+        est[b] = hok ? min(sum, nr * (int64_t)HASH_UMAX) : sum;
+      }
       // the accumulators (R31, R33) emit up to one chunk per warp
       slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)ACC_MAX_WARPS) +
                                2 * (int64_t)min(nlong, PTR_MAX) : 0;
@@ -220,12 +229,13 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
 void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int64_t* seg,
                          const int32_t* nblocks_dev, int64_t max_blocks, int32_t* nzb, int32_t* nze,
                          int64_t* products, int64_t* slots, int32_t* hash_ok, int64_t* ncand,
-                         int64_t* max_products, int64_t* nblocks_out, cudaStream_t st) {
+                         int64_t* max_products, int64_t* nblocks_out, const int32_t* brs, int64_t rows_a,
+                         int64_t* est, cudaStream_t st) {
   if (max_blocks == 0) return;
   const int T = 256, WPB = T / 32;
   k_block_bounds<<<(unsigned)((max_blocks + WPB - 1) / WPB), T, 0, st>>>(
       A.row_ptr, A.col, B.row_ptr, B.col, nseg, seg, nblocks_dev, max_blocks, nzb, nze, products, slots, hash_ok,
-      ncand, max_products, nblocks_out);
+      ncand, max_products, nblocks_out, brs, rows_a, est);
 }
 
 // Canonical-CSR check (reading R3): row_ptr monotone, columns strictly increasing and

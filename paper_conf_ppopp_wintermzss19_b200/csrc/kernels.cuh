@@ -39,7 +39,9 @@ void launch_block_bounds(const CsrView& A, const CsrView& B, int nseg, const int
                          int32_t* blk_hash_ok /* nullable: hash-accumulator candidates (R31) */,
                          int64_t* ncand /* nullable: their count (zeroed by the caller) */,
                          int64_t* max_products /* atomicMax of block products > INT_MAX (zeroed) */,
-                         int64_t* nblocks_out /* nullable: the block count as int64 */, cudaStream_t st);
+                         int64_t* nblocks_out /* nullable: the block count as int64 */,
+                         const int32_t* block_row_starts, int64_t rows_a,
+                         int64_t* est /* nullable: POOL_BOUND region per block (reading R40) */, cudaStream_t st);
 
 // ---- device-wide exclusive scan (scan.cu) --------------------------------------
 // out[i] = sum_{j<i} in[j] for i < n, total -> *total_dev.  tmp needs scan_tmp_elems(n)
@@ -81,6 +83,11 @@ struct EscArgs {
   int64_t* esc_next_small;      // (zeroed)
   int64_t* rows_next;           // adaptive: batch counter of the persistent k_rows (zeroed)
   int32_t rows_batch;           // blocks per k_rows batch, 0: one CTA per block (set by launch_rows)
+  int32_t bound;                // POOL_BOUND (reading R40): warp runs packed by min(row products,
+                                // HASH_UMAX); a block left to AC-ESC whose region is below its
+                                // products is deferred (hash_done = 4) instead of listed
+  const int64_t* region;        // POOL_BOUND: each block's pool region (elements)
+  int64_t* defer;               // POOL_BOUND: [0] deferred blocks, [1] their products (zeroed)
 };
 void launch_esc(const EscArgs& a, bool f64, cudaStream_t st);
 // adaptive alternative (hash.cu, reading R31): must run before launch_esc on the same stream
@@ -93,6 +100,10 @@ void launch_dict(const EscArgs& a, bool f64, cudaStream_t st);
 // others go onto the AC-ESC lists (esc_list / esc_list_small) for launch_esc
 // hash_ran: an accumulator ran before (persistent batches), else one CTA per block
 void launch_rows(const EscArgs& a, bool f64, bool hash_ran, cudaStream_t st);
+// POOL_BOUND second pass (rows.cu, reading R40): flag[b] = products of deferred blocks;
+// after its scan, their regions off[b] = base + scan[b] and the AC-ESC lists
+void launch_defer_flags(const EscArgs& a, int64_t* flag, cudaStream_t st);
+void launch_defer_place(const EscArgs& a, const int64_t* scan, int64_t base, int64_t* off, cudaStream_t st);
 
 // ---- stage 3: chunk ordering, shared rows, merges (merge.cu) --------------------
 struct MergeState {

@@ -77,7 +77,8 @@ struct acspgemm_plan_s {
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan, hdone, esc_list, esc_list_small;
-  DevBuf lgiant, g_lo, g_nsl, g_base, g_pos, g_tcol, g_tval, g_tcnt;   // dense-slice merge (R30): lists, spans, slices
+  DevBuf lgiant, g_lo, g_nsl, g_base, g_pos, g_tcol, g_tval, g_tcnt;
+  DevBuf best, boff, bdef, bdef_scan;   // POOL_BOUND (R40): regions, their scan, deferred flags + scan   // dense-slice merge (R30): lists, spans, slices
   DevBuf trace;                  // acspgemm_set_trace: per block (SM, start, end) x 4 kernels (mpL)
   bool trace_on = false;
   int64_t trace_blocks = 0;
@@ -140,6 +141,26 @@ acspgemm_status ensure(DevBuf& b, size_t bytes) {
     if (s_ != ACSPGEMM_OK) return s_;                   \
   } while (0)
 
+// Grow a buffer to `bytes`, keeping its first `keep` bytes (POOL_BOUND's deferred regions).
+acspgemm_status grow_keep(DevBuf& b, size_t bytes, size_t keep, cudaStream_t st) {
+  if (b.bytes >= bytes) return ACSPGEMM_OK;
+  void* np = nullptr;
+  const size_t want = bytes + bytes / 8;
+  cudaError_t e = cudaMalloc(&np, want);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, "cudaMalloc(" + std::to_string(want) + " bytes): " + cudaGetErrorString(e));
+  }
+  if (keep && b.p) {
+    e = cudaMemcpyAsync(np, b.p, keep, cudaMemcpyDeviceToDevice, st);
+    if (e != cudaSuccess) return set_err(ACSPGEMM_ERR_CUDA, std::string("cudaMemcpyAsync: ") + cudaGetErrorString(e));
+  }
+  if (b.p) cudaFree(b.p);                  // synchronises: the copy is done
+  b.p = np;
+  b.bytes = want;
+  return ACSPGEMM_OK;
+}
+
 // scan_tmp: zero when (re)allocated; the scans leave it zero (scan.cu)
 acspgemm_status ensure_scan_tmp(DevBuf& b, int64_t elems, cudaStream_t st) {
   void* old = b.p;
@@ -187,7 +208,7 @@ int64_t helper_bytes(acspgemm_plan p) {
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->descs, &p->dense, &p->sflag,
                   &p->spos, &p->shared, &p->row_count, &p->row_ptr, &p->scan_tmp, &p->kflag, &p->kpos,
                   &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
-                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->hdone, &p->esc_list, &p->esc_list_small};
+                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->hdone, &p->esc_list, &p->esc_list_small, &p->best, &p->boff, &p->bdef, &p->bdef_scan};
   int64_t t = 0;
   for (DevBuf* b : bs) t += (int64_t)b->bytes;
   return t;
@@ -303,18 +324,26 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->hdone, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->esc_list, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->esc_list_small, sizeof(int32_t) * max_blocks);
+  // POOL_BOUND / AUTO (reading R40): per-block regions bounded by the accumulators' output
+  const bool want_bound = p->opt.pool_mode != ACSPGEMM_POOL_EXACT && p->opt.strategy != ACSPGEMM_STRATEGY_ESC &&
+                          p->opt.strategy != ACSPGEMM_STRATEGY_DICT;
+  if (want_bound) {
+    ACS_ENSURE(p->best, sizeof(int64_t) * max_blocks);
+    ACS_ENSURE(p->boff, sizeof(int64_t) * max_blocks);
+  }
   const int64_t tmp_n = scan_tmp_elems(std::max<int64_t>(max_blocks, A->rows) * 2 + 1024);
   ACS_ENSURE_SCAN_TMP(p->scan_tmp, tmp_n, st);
   ACS_ENSURE(p->row_count, sizeof(int32_t) * A->rows);
   int32_t* nblocks_dev = reinterpret_cast<int32_t*>(scal + 20);
   // scal words: 0 products, 1 slots, 2 nblocks, 3 ncand / total chunks, 4 max block
-  // products / shared rows, 5 chunk elements, 6 hash blocks, 7 dict blocks, 8..14 merge
-  // class counts, 15 k_rows blocks, 16 nnz(C), 20 nblocks (int32), 24-25 dense slices,
-  // 26 k_rows batches, 28-31 AC-ESC lists.  The counters are zeroed by k_segments, the
+  // products / shared rows, 5 bounded pool / chunk elements, 6 hash blocks, 7 dict
+  // blocks, 8..14 merge class counts, 15 k_rows blocks, 16 nnz(C), 17-18 deferred blocks
+  // and their products, 20 nblocks (int32), 23-25 dense slices, 26 k_rows batches, 28-31
+  // AC-ESC lists.  The counters are zeroed by k_segments, the
   // first kernel (with err), and k_glb zeroes the per-row counters: no memset launches.
   ZeroList zero{};
   zero.p[0] = scal + 3; zero.n[0] = 2;
-  zero.p[1] = scal + 6; zero.n[1] = 10;
+  zero.p[1] = scal + 6; zero.n[1] = 13;
   zero.p[2] = scal + 26; zero.n[2] = 6;
   zero.p[3] = reinterpret_cast<int64_t*>(p->err.p); zero.n[3] = 2;
   launch_segments(Av, nseg, explicit_rows, ptr<int64_t>(p->seg), nblocks_dev, st, zero);
@@ -324,15 +353,19 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   launch_block_bounds(Av, Bv, nseg, ptr<int64_t>(p->seg), nblocks_dev, max_blocks, ptr<int32_t>(p->nzb),
                       ptr<int32_t>(p->nze), ptr<int64_t>(p->bprod), ptr<int64_t>(p->bslot),
                       p->opt.strategy != ACSPGEMM_STRATEGY_ESC ? ptr<int32_t>(p->hdone) : nullptr, scal + 3, scal + 4,
-                      scal + 2, st);
+                      scal + 2, ptr<int32_t>(p->brs), A->rows, want_bound ? ptr<int64_t>(p->best) : nullptr, st);
   tl_launches += 1;
   launch_scan_i64(ptr<int64_t>(p->bprod), ptr<int64_t>(p->pool_off), max_blocks, scal + 0, ptr<int64_t>(p->scan_tmp), st);
   launch_scan_i64(ptr<int64_t>(p->bslot), ptr<int64_t>(p->desc_off), max_blocks, scal + 1, ptr<int64_t>(p->scan_tmp), st);
   tl_launches += 2;
+  if (want_bound) {
+    launch_scan_i64(ptr<int64_t>(p->best), ptr<int64_t>(p->boff), max_blocks, scal + 5, ptr<int64_t>(p->scan_tmp), st);
+    tl_launches += 1;
+  }
   ACS_CUDA(cudaGetLastError());
   // segment boundaries (for info) ride along with the first read-back (replay: unchanged)
-  if ((s = sync_read(p, scal, 5, st, p->seg.p, p->h_scal + H_SEG_INFO, (int)sizeof(int64_t) * (nseg + 1))) !=
-      ACSPGEMM_OK)
+  if ((s = sync_read(p, scal, want_bound ? 6 : 5, st, p->seg.p, p->h_scal + H_SEG_INFO,
+                     (int)sizeof(int64_t) * (nseg + 1))) != ACSPGEMM_OK)
     return s;
   const int64_t products = p->h_scal[0], slots = p->h_scal[1], nblocks = p->h_scal[2], ncand = p->h_scal[3];
   if (p->h_scal[4] > 0)
@@ -342,12 +375,18 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   p->info.nblocks = nblocks;
   p->info.nsegments = nseg;
   for (int i = 0; i <= nseg; ++i) p->info.segment_rows[i] = p->h_scal[H_SEG_INFO + i];
-  const int64_t pool_bytes = products * (4 + vbytes);
+  const int64_t bound_elems = want_bound ? p->h_scal[5] : products;
+  const bool over_limit = p->opt.pool_limit_bytes && (size_t)(products * (4 + vbytes)) > p->opt.pool_limit_bytes;
+  const bool use_bound = want_bound && (p->opt.pool_mode == ACSPGEMM_POOL_BOUND || over_limit);
+  const int64_t pool_elems = use_bound ? bound_elems : products;
+  const int64_t pool_bytes = pool_elems * (4 + vbytes);
   if (p->opt.pool_limit_bytes && (size_t)pool_bytes > p->opt.pool_limit_bytes)
-    return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, "exact chunk-pool bound " + std::to_string(pool_bytes) +
-                                                   " B exceeds pool_limit_bytes");
-  ACS_ENSURE(p->pool_col, sizeof(int32_t) * products);
-  ACS_ENSURE(p->pool_val, (size_t)vbytes * products);
+    return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, std::string(use_bound ? "bounded" : "exact") + " chunk-pool size " +
+                                                   std::to_string(pool_bytes) + " B exceeds pool_limit_bytes");
+  p->info.pool_mode = use_bound ? ACSPGEMM_POOL_BOUND : ACSPGEMM_POOL_EXACT;
+  p->info.ndeferred_blocks = 0;
+  ACS_ENSURE(p->pool_col, sizeof(int32_t) * pool_elems);
+  ACS_ENSURE(p->pool_val, (size_t)vbytes * pool_elems);
   ACS_ENSURE(p->descs, sizeof(ChunkDesc) * slots);
   // scans later run over up to `slots` chunks / shared rows
   ACS_ENSURE_SCAN_TMP(p->scan_tmp, scan_tmp_elems(std::max<int64_t>(std::max(max_blocks, A->rows), slots) + 1), st);
@@ -362,7 +401,10 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.blk_nz_begin = ptr<int32_t>(p->nzb);
   ea.blk_nz_end = ptr<int32_t>(p->nze);
   ea.block_row_starts = ptr<int32_t>(p->brs);
-  ea.pool_off = ptr<int64_t>(p->pool_off);
+  ea.pool_off = use_bound ? ptr<int64_t>(p->boff) : ptr<int64_t>(p->pool_off);
+  ea.bound = use_bound ? 1 : 0;
+  ea.region = use_bound ? ptr<int64_t>(p->best) : nullptr;
+  ea.defer = scal + 17;
   ea.desc_off = ptr<int64_t>(p->desc_off);
   ea.pool_col = ptr<int32_t>(p->pool_col);
   ea.pool_val = p->pool_val.p;
@@ -427,6 +469,37 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   tl_launches += nblocks > 0 ? 1 : 0;
   ea.trace = nullptr;
   ACS_CUDA(cudaGetLastError());
+  if (use_bound) {
+    // POOL_BOUND (reading R40): candidates that ended in AC-ESC were deferred; their
+    // exact regions are appended to the pool (grown by a copy) and AC-ESC runs on them
+    if ((s = sync_read(p, scal + 17, 2, st)) != ACSPGEMM_OK) return s;
+    const int64_t ndef = p->h_scal[0], def_products = p->h_scal[1];
+    p->info.ndeferred_blocks = ndef;
+    if (ndef > 0) {
+      const int64_t total = bound_elems + def_products;
+      if (p->opt.pool_limit_bytes && (size_t)(total * (4 + vbytes)) > p->opt.pool_limit_bytes)
+        return set_err(ACSPGEMM_ERR_OUT_OF_MEMORY, "bounded chunk pool plus the deferred blocks' exact bounds (" +
+                                                       std::to_string(total * (4 + vbytes)) + " B) exceeds pool_limit_bytes");
+      if ((s = grow_keep(p->pool_col, sizeof(int32_t) * total, sizeof(int32_t) * bound_elems, st)) != ACSPGEMM_OK)
+        return s;
+      if ((s = grow_keep(p->pool_val, (size_t)vbytes * total, (size_t)vbytes * bound_elems, st)) != ACSPGEMM_OK)
+        return s;
+      ea.pool_col = ptr<int32_t>(p->pool_col);
+      ea.pool_val = p->pool_val.p;
+      ACS_ENSURE(p->bdef, sizeof(int64_t) * max_blocks);
+      ACS_ENSURE(p->bdef_scan, sizeof(int64_t) * max_blocks);
+      ACS_CUDA(cudaMemsetAsync(scal + 28, 0, 4 * sizeof(int64_t), st));
+      launch_defer_flags(ea, ptr<int64_t>(p->bdef), st);
+      launch_scan_i64(ptr<int64_t>(p->bdef), ptr<int64_t>(p->bdef_scan), nblocks, scal + 19, ptr<int64_t>(p->scan_tmp),
+                      st);
+      launch_defer_place(ea, ptr<int64_t>(p->bdef_scan), bound_elems, ptr<int64_t>(p->boff), st);
+      acs_launch_esc_small(&ea, p->f64, st);
+      launch_esc(ea, p->f64, st);
+      tl_launches += 5;
+      ACS_CUDA(cudaGetLastError());
+      p->info.pool_bytes = (int64_t)(p->pool_col.bytes + p->pool_val.bytes);
+    }
+  }
 
   // ------------------------------------------------------------ MCC -----------
   record(p, S_MCC, st);
@@ -782,6 +855,7 @@ void acspgemm_options_default(acspgemm_options* opt) {
   opt->collect_stage_times = 0;
   opt->num_segments = DEFAULT_SEGMENTS;
   opt->strategy = ACSPGEMM_STRATEGY_ADAPTIVE;
+  opt->pool_mode = ACSPGEMM_POOL_EXACT;
 }
 
 acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options* opt) {
@@ -823,7 +897,7 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
                   &p->mtscan, &p->group_of, &p->gstart, &p->merge_col, &p->merge_val, &p->cur_first,
                   &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->lgiant, &p->g_lo, &p->g_nsl,
                   &p->g_base, &p->g_pos, &p->g_tcol, &p->g_tval, &p->g_tcnt, &p->hdone, &p->esc_list,
-                  &p->esc_list_small, &p->trace};
+                  &p->esc_list_small, &p->trace, &p->best, &p->boff, &p->bdef, &p->bdef_scan};
   for (DevBuf* b : bs) free_buf(*b);
   for (auto& pb : p->bp) for (DevBuf& b : pb) free_buf(b);
   if (p->gexec) cudaGraphExecDestroy(p->gexec);

@@ -50,7 +50,7 @@ struct RowsSmem {
     } l;
   } u;
   int wrow[ROWS_WARPS + 1];
-  int wout[ROWS_WARPS][5];
+  int wout[ROWS_WARPS][6];
   alignas(8) int scratch[40];
   int flag;
   int batch[32];                 // the current batch's blocks no accumulator finished
@@ -59,6 +59,13 @@ struct RowsSmem {
 
 // A block left to AC-ESC: onto the big- or small-tile list (reading R32).
 __device__ __forceinline__ void rows_give_up(const EscArgs& a, int b) {
+  if (a.bound && a.region[b] < a.blk_products[b]) {
+    // POOL_BOUND: AC-ESC needs the block's exact bound; deferred to a second pass (R40)
+    a.hash_done[b] = 4;
+    atomicAdd(reinterpret_cast<unsigned long long*>(a.defer), 1ull);
+    atomicAdd(reinterpret_cast<unsigned long long*>(a.defer + 1), (unsigned long long)a.blk_products[b]);
+    return;
+  }
   const bool small = a.esc_list_small && a.blk_products[b] <= CAP_SMALL;
   int64_t* cnt = small ? a.esc_count_small : a.esc_count;
   int32_t* list = small ? a.esc_list_small : a.esc_list;
@@ -86,7 +93,8 @@ __device__ __forceinline__ void rows_block(RowsSmem<T>& S, const EscArgs& a, con
   split_rows<ROWS_WARPS>(S.wd, S.row_first, nrows, total, S.wrow);
   __syncthreads();
   const int rlo = S.wrow[w], rhi = S.wrow[w + 1];
-  const int64_t wbase = a.pool_off[b] + (rlo < nrows ? S.wd[S.row_first[rlo]] : 0);
+  const int wrel = warp_out_base(a, S.wd, S.row_first, rlo, nrows, lane);
+  const int64_t wbase = a.pool_off[b] + wrel;
   T* pval = reinterpret_cast<T*>(a.pool_val);
   int32_t* pcol = a.pool_col;
   int(*lc)[THREADS] = S.u.l.col;
@@ -186,6 +194,7 @@ __device__ __forceinline__ void rows_block(RowsSmem<T>& S, const EscArgs& a, con
     S.wout[w][2] = last_row;
     S.wout[w][3] = first_count;
     S.wout[w][4] = last_count;
+    S.wout[w][5] = wrel;
   }
   __syncthreads();
   if (tid == 0) trace_block(a.trace, b, t_start);
@@ -236,6 +245,33 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
       __syncthreads();                   // shared memory is reused by the next block
     }
   }
+}
+
+// POOL_BOUND second pass (reading R40): the deferred blocks (hash_done == 4) get regions of
+// their exact product bound appended to the pool, in block order (a scan), and go onto
+// the AC-ESC lists (big / small tile).
+__global__ void k_defer_flags(const int32_t* __restrict__ hash_done, const int64_t* __restrict__ prod, int n,
+                              int64_t* __restrict__ flag) {
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b < n) flag[b] = hash_done[b] == 4 ? prod[b] : 0;
+}
+
+__global__ void k_defer_place(EscArgs a, const int64_t* __restrict__ scan, int64_t base, int64_t* __restrict__ off) {
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= a.nblocks || a.hash_done[b] != 4) return;
+  off[b] = base + scan[b];
+  const bool small = a.esc_list_small && a.blk_products[b] <= CAP_SMALL;
+  int64_t* cnt = small ? a.esc_count_small : a.esc_count;
+  int32_t* list = small ? a.esc_list_small : a.esc_list;
+  list[atomicAdd(reinterpret_cast<unsigned long long*>(cnt), 1ull)] = b;
+}
+
+void launch_defer_flags(const EscArgs& a, int64_t* flag, cudaStream_t st) {
+  if (a.nblocks > 0) k_defer_flags<<<(a.nblocks + 255) / 256, 256, 0, st>>>(a.hash_done, a.blk_products, a.nblocks, flag);
+}
+
+void launch_defer_place(const EscArgs& a, const int64_t* scan, int64_t base, int64_t* off, cudaStream_t st) {
+  if (a.nblocks > 0) k_defer_place<<<(a.nblocks + 255) / 256, 256, 0, st>>>(a, scan, base, off);
 }
 
 template <typename T>

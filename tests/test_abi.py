@@ -28,7 +28,7 @@ def test_library_exports_every_header_symbol():
 def test_host_only_entry_points():
     import paper_conf_ppopp_wintermzss19_b200 as pkg
     lib = pkg.load()
-    assert lib.acspgemm_abi_version() == 1
+    assert lib.acspgemm_abi_version() == 2
     assert pkg.const("NPB") == 512 and pkg.const("CAP") == 2048 and pkg.const("KEEP") == 4 * pkg.const("THREADS")
     assert lib.acspgemm_const(99) == -1
     assert lib.acspgemm_status_string(0) == b"ok"
