@@ -205,6 +205,49 @@ def test_hash_stencil_square_exact(cuda_available):
 
 
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_hash_row_reuse_sentinel_corners(dt, cuda_available):
+    """Row-relative keys (reading R41): a warp keeps its keys from row to row and a row
+    whose touched slots equal the previous row's reuses its column order.  A value that
+    reads like an untouched slot after it was touched -- a column whose products are all
+    -0.0, or (fp64) a sum in (-2^-1042, 0) that shares -0.0's high word -- must not
+    corrupt the row: such blocks go to AC-ESC.  The 27-point stencil's boundary rows
+    (subsets of the interior pattern), a few random rows between translate-equal ones,
+    and values equal to the oracle everywhere; the same bits run to run."""
+    A = poisson3d_27pt(14)
+    B = poisson3d_27pt(14)
+    rng = np.random.default_rng(41)
+    aval = np.abs(rng.uniform(0.5, 1.5, A.nnz))
+    bval = rng.uniform(-1, 1, B.nnz)
+    bval[np.isin(B.col, [300, 301, 1500])] = -0.0          # all products -0.0 (A > 0)
+    if dt == np.float64:
+        bval[np.isin(B.col, [900, 2200])] = -1e-321        # sums share -0.0's high word
+    A = synth_csr(A, aval)
+    B = synth_csr(B, bval)
+    out, info = run(A, B, dt)
+    check(out, A, B, dt)
+    assert info["nhash_blocks"] > 0
+    out2, _ = run(A, B, dt)
+    assert digest(*out) == digest(*out2)
+    # rows of a banded pattern with random rows in between (reuse on, off, on again)
+    n = 3000
+    r, c = [], []
+    for i in range(n):
+        cols = np.arange(i - 10, i + 11) if i % 50 else rng.choice(n, 21, replace=False)
+        cols = np.unique(np.clip(cols, 0, n - 1))
+        r += [i] * len(cols)
+        c += cols.tolist()
+    M = from_coo(n, n, np.array(r), np.array(c), rng.uniform(-1, 1, len(r)))
+    out, info = run(M, M, dt)
+    check(out, M, M, dt)
+    assert info["nhash_blocks"] > 0
+
+
+def synth_csr(M, val):
+    from synth import CSR
+    return CSR(M.rows, M.cols, M.row_ptr, M.col, np.asarray(val, dtype=M.val.dtype))
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
 def test_low_compaction_rows_go_to_esc(dt, cuda_available):
     """Rows whose products hardly compact (random columns: adjacent entries' B rows share
     almost no columns) are not hash candidates; AC-ESC computes them."""
