@@ -2,6 +2,7 @@
 // reading R31; dict.cu, reading R33): exact IEEE product/sum and Fetch A.
 #pragma once
 #include <climits>
+#include <type_traits>
 #include "kernels.cuh"
 
 namespace acs {
@@ -10,6 +11,14 @@ __device__ __forceinline__ float vmul(float x, float y) { return __fmul_rn(x, y)
 __device__ __forceinline__ double vmul(double x, double y) { return __dmul_rn(x, y); }
 __device__ __forceinline__ float vadd(float x, float y) { return __fadd_rn(x, y); }
 __device__ __forceinline__ double vadd(double x, double y) { return __dadd_rn(x, y); }
+
+// A compacted entry and its A value in one 16-byte record (k_hash reads a wave's entry
+// with one shared-memory load); fetch_block fills it when E is EntA<T> (a_val unused).
+template <typename T>
+struct alignas(16) EntA {
+  int x, y;   // B row start, B row length
+  T a;        // the A value
+};
 
 // Block-wide exclusive prefix sum for a CTA of NT threads (the fixed shuffle tree of
 // common.cuh's block_exclusive_sum).  `scratch` needs NT/32 + 1 elements.  Two
@@ -153,9 +162,13 @@ __device__ __forceinline__ bool fetch_block(const EscArgs& a, int b, int* rp_cac
       row_of[lr] = row[j];
     }
     if (len[j] > 0) {
-      ent[ci].x = bst[j];
-      ent[ci].y = len[j];
-      a_val[ci] = av[j];
+      if constexpr (std::is_same<E, EntA<T>>::value) {
+        ent[ci] = EntA<T>{bst[j], len[j], av[j]};
+      } else {
+        ent[ci].x = bst[j];
+        ent[ci].y = len[j];
+        a_val[ci] = av[j];
+      }
       wd[ci] = pex;
     }
     ex += f[j] + ((len[j] > 0) << 16);

@@ -67,11 +67,10 @@ constexpr int HASH_WARPS = ACS_HASH_WARPS;   // warps per CTA; each emits one ch
 constexpr int ACC_MAX_WARPS = 8;             // most warps (= chunks) an accumulator uses per block (k_dict)
 static_assert(HASH_WARPS <= ACC_MAX_WARPS, "chunk slots per block (k_block_bounds)");
 constexpr int HASH_THREADS = 32 * HASH_WARPS;
-#ifndef ACS_HASH_TBITS
-#define ACS_HASH_TBITS 9
+#ifndef ACS_HASH_T
+#define ACS_HASH_T 512
 #endif
-constexpr int HASH_TBITS = ACS_HASH_TBITS;   // log2 of the table slots per warp
-constexpr int HASH_T = 1 << HASH_TBITS;      // table slots per warp
+constexpr int HASH_T = ACS_HASH_T;           // table slots per warp (a multiple of 32)
 constexpr int HASH_UMAX = HASH_T / 2;        // max distinct columns of a row (load <= 1/2)
 #ifndef ACS_HASH_PROWMAX
 #define ACS_HASH_PROWMAX 2048
