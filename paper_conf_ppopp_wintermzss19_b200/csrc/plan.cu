@@ -420,6 +420,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.esc_count = scal + 28;
   ea.esc_next = scal + 29;
   ea.rows_next = scal + 26;
+  ea.hash_next = scal + 27;
   ea.blk_products = ptr<int64_t>(p->bprod);
   ea.esc_list_small = nullptr;
   ea.trace = nullptr;
