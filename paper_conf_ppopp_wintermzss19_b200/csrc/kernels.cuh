@@ -83,6 +83,8 @@ struct EscArgs {
   int64_t* esc_next_small;      // (zeroed)
   int64_t* rows_next;           // adaptive: batch counter of the persistent k_rows (zeroed)
   int64_t* hash_next;           // adaptive: block counter of the persistent k_hash (zeroed)
+  int32_t* rows_list;           // adaptive: blocks k_hash saw and did not finish, for k_rows
+  int64_t* rows_list_count;     // (zeroed) their number; nullptr: k_rows scans hash_done
   int32_t rows_batch;           // blocks per k_rows batch, 0: one CTA per block (set by launch_rows)
   int32_t bound;                // POOL_BOUND (reading R40): warp runs packed by min(row products,
                                 // HASH_UMAX); a block left to AC-ESC whose region is below its

@@ -73,7 +73,7 @@ struct acspgemm_plan_s {
   int nseg_explicit = 0;
   int64_t seg_rows_explicit[MAX_SEGMENTS + 1];
   // buffers
-  DevBuf seg, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base;
+  DevBuf seg, scal, brs, nzb, nze, bprod, bslot, pool_off, desc_off, nchunks, chunk_base, rows_list;
   DevBuf pool_col, pool_val, descs, dense, sflag, spos, shared, row_count, row_ptr, scan_tmp;
   DevBuf kflag, kpos, lmulti, lpath, lsearch, lpair, mscan, mtscan, group_of, gstart, merge_col, merge_val;
   DevBuf cur_first, cur_last, err, bused, bused_scan, hdone, esc_list, esc_list_small;
@@ -208,7 +208,7 @@ int64_t helper_bytes(acspgemm_plan p) {
                   &p->pool_off, &p->desc_off, &p->nchunks, &p->chunk_base, &p->descs, &p->dense, &p->sflag,
                   &p->spos, &p->shared, &p->row_count, &p->row_ptr, &p->scan_tmp, &p->kflag, &p->kpos,
                   &p->lmulti, &p->lpath, &p->lsearch, &p->lpair, &p->mscan, &p->mtscan, &p->group_of, &p->gstart,
-                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->hdone, &p->esc_list, &p->esc_list_small, &p->best, &p->boff, &p->bdef, &p->bdef_scan};
+                  &p->merge_col, &p->merge_val, &p->cur_first, &p->cur_last, &p->err, &p->bused, &p->bused_scan, &p->hdone, &p->esc_list, &p->esc_list_small, &p->rows_list, &p->best, &p->boff, &p->bdef, &p->bdef_scan};
   int64_t t = 0;
   for (DevBuf* b : bs) t += (int64_t)b->bytes;
   return t;
@@ -324,6 +324,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ACS_ENSURE(p->hdone, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->esc_list, sizeof(int32_t) * max_blocks);
   ACS_ENSURE(p->esc_list_small, sizeof(int32_t) * max_blocks);
+  ACS_ENSURE(p->rows_list, sizeof(int32_t) * max_blocks);
   // POOL_BOUND / AUTO (reading R40): per-block regions bounded by the accumulators' output
   const bool want_bound = p->opt.pool_mode != ACSPGEMM_POOL_EXACT && p->opt.strategy != ACSPGEMM_STRATEGY_ESC &&
                           p->opt.strategy != ACSPGEMM_STRATEGY_DICT;
@@ -338,13 +339,14 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   // scal words: 0 products, 1 slots, 2 nblocks, 3 ncand / total chunks, 4 max block
   // products / shared rows, 5 bounded pool / chunk elements, 6 hash blocks, 7 dict
   // blocks, 8..14 merge class counts, 15 k_rows blocks, 16 nnz(C), 17-18 deferred blocks
-  // and their products, 20 nblocks (int32), 23-25 dense slices, 26 k_rows batches, 28-31
+  // and their products, 20 nblocks (int32), 21 k_rows list, 23-25 dense slices, 26 k_rows
+  // batches, 27 k_hash blocks, 28-31
   // AC-ESC lists.  The counters are zeroed by k_segments, the
   // first kernel (with err), and k_glb zeroes the per-row counters: no memset launches.
   ZeroList zero{};
   zero.p[0] = scal + 3; zero.n[0] = 2;
   zero.p[1] = scal + 6; zero.n[1] = 13;
-  zero.p[2] = scal + 26; zero.n[2] = 6;
+  zero.p[2] = scal + 21; zero.n[2] = 11;
   zero.p[3] = reinterpret_cast<int64_t*>(p->err.p); zero.n[3] = 2;
   launch_segments(Av, nseg, explicit_rows, ptr<int64_t>(p->seg), nblocks_dev, st, zero);
   tl_launches += 1;
@@ -421,6 +423,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   ea.esc_next = scal + 29;
   ea.rows_next = scal + 26;
   ea.hash_next = scal + 27;
+  ea.rows_list = nullptr;
+  ea.rows_list_count = nullptr;
   ea.blk_products = ptr<int64_t>(p->bprod);
   ea.esc_list_small = nullptr;
   ea.trace = nullptr;
@@ -451,6 +455,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   record(p, S_DICTEND, st);
   if (ea.hash_done && ncand > 0) {
     ea.trace = trace_of(0);
+    ea.rows_list = ptr<int32_t>(p->rows_list);   // k_hash lists the blocks it leaves for k_rows
+    ea.rows_list_count = scal + 21;
     launch_hash(ea, p->f64, st);         // blocks k_dict left (reading R31)
     tl_launches += nblocks > 0 ? 1 : 0;
   }

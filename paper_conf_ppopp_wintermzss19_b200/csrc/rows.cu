@@ -230,16 +230,19 @@ __global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
       if (tid == 0)
         base = (int)atomicAdd(reinterpret_cast<unsigned long long*>(a.rows_next), (unsigned long long)a.rows_batch);
       base = __shfl_sync(0xffffffffu, base, 0);
-      const int b = base + tid;
-      const bool need = tid < a.rows_batch && b < a.nblocks && a.hash_done[b] == 0;
+      // after k_hash: its list of the blocks it left; otherwise every block, by flag
+      const int limit = a.rows_list ? (int)*a.rows_list_count : a.nblocks;
+      const int i = base + tid;
+      const int b = a.rows_list ? (i < limit ? a.rows_list[i] : 0) : i;
+      const bool need = tid < a.rows_batch && i < limit && a.hash_done[b] == 0;
       const unsigned m = __ballot_sync(0xffffffffu, need);
       if (need) S.batch[__popc(m & ((1u << tid) - 1u))] = b;
-      if (tid == 0) { S.nbatch = __popc(m); S.bbase = base; }
+      if (tid == 0) { S.nbatch = __popc(m); S.bbase = base < limit ? 0 : 1; }
     }
     __syncthreads();
     const int bbase = S.bbase, n = S.nbatch;
     __syncthreads();                     // read before warp 0 overwrites them (n == 0)
-    if (bbase >= a.nblocks) break;
+    if (bbase) break;                    // past the last block
     for (int k = 0; k < n; ++k) {
       rows_block<T>(S, a, S.batch[k]);
       __syncthreads();                   // shared memory is reused by the next block

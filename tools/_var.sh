@@ -1,6 +1,6 @@
 mkdir -p gpurun_out; rm -f gpurun_out/var.txt
 L=paper_conf_ppopp_wintermzss19_b200
-for v in "" _t384 _t384c _t256 _t256b6; do
+for v in "" _w4 _w2; do
   for dt in f64 f32; do
     ACSPGEMM_LIB=$PWD/$L/libacspgemm$v.so python tools/strat_cmp.py cfg2 $dt adaptive 10 2>&1 | head -1 | sed "s/^/var$v /" >> gpurun_out/var.txt
   done
