@@ -242,6 +242,29 @@ def test_hash_row_reuse_sentinel_corners(dt, cuda_available):
     assert info["nhash_blocks"] > 0
 
 
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_hash_stale_keys_clear_and_rerun(dt, cuda_available):
+    """Rows whose row-relative patterns drift (row i's columns are [12i, 12i + 126): the
+    relative keys shift by 11 per row) fill a warp's table with earlier rows' keys; after
+    about 12 rows a row would push it past HASH_UMAX keys, clears the table and runs again
+    (reading R41).  Every block stays with the hash accumulator and C equals the
+    oracle's.  (Rows of 9 entries: the candidate test samples adjacent entries 63 apart,
+    which rows of 8 would put on row boundaries.)"""
+    n = 3000
+    r = np.repeat(np.arange(n), 9)
+    c = (np.arange(n)[:, None] + np.arange(9)[None, :]).ravel()
+    rng = np.random.default_rng(17)
+    A = from_coo(n, n + 9, r, c, rng.uniform(-1, 1, len(r)))
+    rb = np.repeat(np.arange(n + 9), 30)
+    cb = (12 * np.arange(n + 9)[:, None] + np.arange(30)[None, :]).ravel()
+    B = from_coo(n + 9, 12 * (n + 9) + 30, rb, cb, rng.uniform(-1, 1, len(rb)))
+    out, info = run(A, B, dt)
+    check(out, A, B, dt)
+    assert info["nhash_blocks"] == info["nblocks"]
+    out2, _ = run(A, B, dt)
+    assert digest(*out) == digest(*out2)
+
+
 def synth_csr(M, val):
     from synth import CSR
     return CSR(M.rows, M.cols, M.row_ptr, M.col, np.asarray(val, dtype=M.val.dtype))
