@@ -515,15 +515,10 @@ __global__ void __launch_bounds__(THREADS, ESC_MIN_BLOCKS) k_esc(EscArgs a) {
 template <typename T>
 static void launch_esc_t(const EscArgs& a, cudaStream_t st) {
   const size_t smem = sizeof(EscSmem<T>);
-  cudaFuncSetAttribute(k_esc<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  static ResidentCache rc;
+  const int resident = resident_ctas(rc, k_esc<T>, THREADS, smem);   // also sets the smem limit
   int grid = a.nblocks;
-  if (a.hash_done) {
-    int dev = 0, sms = 148, per = ESC_MIN_BLOCKS;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_esc<T>, THREADS, smem);
-    grid = std::min<int>(a.nblocks, std::max(1, sms * std::max(per, 1)));
-  }
+  if (a.hash_done) grid = std::min<int>(a.nblocks, std::max(1, resident));
   k_esc<T><<<grid, THREADS, smem, st>>>(a);
 }
 

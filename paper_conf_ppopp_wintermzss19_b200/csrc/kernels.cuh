@@ -217,6 +217,28 @@ void launch_read_back2(const void* src1, void* mapped_dst1, int nbytes1, const v
 // p[i] += off for i < n (row pointers of a row piece placed after earlier pieces)
 void launch_add_offset(int32_t* p, int64_t n, int32_t off, cudaStream_t st);
 
+// Resident CTAs of `kern` on the current device (SMs x CTAs per SM at `threads` threads and
+// `smem` dynamic shared memory), worked out once per device per kernel (the host calls
+// sit between a read-back and the next launch: on the critical path of small
+// multiplies); raises the kernel's dynamic shared-memory limit to `smem` the same once.
+struct ResidentCache {
+  int grid[16] = {0};
+};
+template <typename K>
+inline int resident_ctas(ResidentCache& c, K kern, int threads, size_t smem) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int* slot = (dev >= 0 && dev < 16) ? &c.grid[dev] : nullptr;
+  if (slot && *slot > 0) return *slot;
+  cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  int sms = 148, per = 1;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, threads, smem);
+  const int g = sms * (per > 0 ? per : 1);
+  if (slot) *slot = g;
+  return g;
+}
+
 // ---- validation ----------------------------------------------------------------
 void launch_validate(const CsrView& M, int32_t* bad_flag, cudaStream_t st);
 

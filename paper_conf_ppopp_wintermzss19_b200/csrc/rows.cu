@@ -280,14 +280,10 @@ void launch_defer_place(const EscArgs& a, const int64_t* scan, int64_t base, int
 template <typename T>
 static void launch_rows_t(const EscArgs& a, bool hash_ran, cudaStream_t st) {
   const size_t smem = sizeof(RowsSmem<T>);
-  cudaFuncSetAttribute(k_rows<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  int dev = 0, sms = 148, per = 1;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_rows<T>, THREADS, smem);
+  static ResidentCache rc;
   // batches of up to ROWS_BATCH blocks, at least ~16 per CTA (a short tail), one block
   // per batch when there are fewer blocks than CTAs
-  const int64_t slots = (int64_t)sms * std::max(per, 1);
+  const int64_t slots = resident_ctas(rc, k_rows<T>, THREADS, smem);   // also sets the smem limit
   EscArgs b = a;
   if (!hash_ran) {                       // no accumulator ran: one CTA per block
     b.rows_batch = 0;
