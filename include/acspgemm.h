@@ -101,13 +101,15 @@ typedef struct {
                                 ACSPGEMM_STRATEGY_DICT: block dictionary (R33), hash, AC-ESC.
                                 ADAPTIVE, HASH and DICT give the same results bit for bit. */
   int pool_mode;             /* chunk-pool sizing (L556, L580; reading R40):
-                                ACSPGEMM_POOL_EXACT (default): every block owns its exact product
-                                bound, products x (4 + value size) in all -- no overflow path;
-                                ACSPGEMM_POOL_BOUND: a hash-accumulator candidate block owns
-                                min(products, rows x 256) (the accumulators' output bound); a
-                                candidate that ends in AC-ESC is deferred and run after the first
-                                pass in a region of its exact bound appended to the pool (one more
-                                read-back; the pool grows by a copy).  Same bytes of C;
+                                ACSPGEMM_POOL_BOUND (default): a hash-accumulator candidate block
+                                owns min(products, rows x HASH_UBOUND = 192) (the accumulators'
+                                output bound; in this mode a row of more distinct columns sends
+                                its block to AC-ESC); a candidate that ends in AC-ESC is deferred
+                                and run after the first pass in a region of its exact bound
+                                appended to the pool (one more read-back; the pool grows by a
+                                copy); other blocks own their exact product bound.  Same bytes of C;
+                                ACSPGEMM_POOL_EXACT: every block owns its exact product bound,
+                                products x (4 + value size) in all -- no overflow path;
                                 ACSPGEMM_POOL_AUTO: EXACT when the exact bound fits
                                 pool_limit_bytes (or there is no limit), else BOUND.
                                 The DICT strategy always uses EXACT. */

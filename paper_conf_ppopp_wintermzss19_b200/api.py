@@ -91,7 +91,7 @@ class Plan:
     """A reusable multiply plan (owns the chunk pool and helper memory)."""
 
     def __init__(self, pool_limit_bytes: int = 0, validate: bool = False, stage_times: bool = False,
-                 num_segments: int = 8, strategy: str = "adaptive", pool_mode: str = "exact"):
+                 num_segments: int = 8, strategy: str = "adaptive", pool_mode: str = "bound"):
         """strategy: "adaptive" (hash accumulator per candidate block, per-row accumulator
         for blocks of short rows, AC-ESC fallback; readings R31, R34), "hash" (the same path;
         kept for the round-1 API), "dict" (column dictionary first, reading R33) -- these three give the

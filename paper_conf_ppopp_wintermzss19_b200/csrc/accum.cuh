@@ -205,14 +205,14 @@ __device__ __forceinline__ void split_rows(const int* wd, const int* row_first, 
 // block in *counter (info only).  Thread 0.
 // Where (relative to the block's pool region) the warp owning rows [rlo, ..) writes: exact
 // pools: after the products of the rows before it; POOL_BOUND (reading R40): after
-// sum min(products, HASH_UMAX) over them -- the accumulators' output bound, so the runs
+// sum min(products, HASH_UBOUND) over them -- the accumulators' output bound, so the runs
 // pack into min(products, rows x HASH_UMAX).  All lanes of the warp call it.
 __device__ __forceinline__ int warp_out_base(const EscArgs& a, const int* wd, const int* row_first, int rlo,
                                              int nrows, int lane) {
   if (rlo >= nrows) return 0;
   if (!a.bound) return wd[row_first[rlo]];
   int s = 0;
-  for (int r = lane; r < rlo; r += 32) s += min(wd[row_first[r + 1]] - wd[row_first[r]], HASH_UMAX);
+  for (int r = lane; r < rlo; r += 32) s += min(wd[row_first[r + 1]] - wd[row_first[r]], HASH_UBOUND);
   return __reduce_add_sync(0xffffffffu, s);
 }
 

@@ -72,6 +72,14 @@ constexpr int HASH_THREADS = 32 * HASH_WARPS;
 #endif
 constexpr int HASH_T = ACS_HASH_T;           // table slots per warp (a multiple of 32)
 constexpr int HASH_UMAX = HASH_T / 2;        // max distinct columns of a row (load <= 1/2)
+#ifndef ACS_HASH_UBOUND
+#define ACS_HASH_UBOUND 192
+#endif
+// POOL_BOUND (reading R40): an accumulator row's output cap, so a candidate block's region
+// is sum min(row products, HASH_UBOUND); a row with more distinct columns sends its block
+// to AC-ESC (deferred, exact region) in that mode only
+constexpr int HASH_UBOUND = ACS_HASH_UBOUND;
+static_assert(HASH_UBOUND <= HASH_UMAX, "the bound cap cannot exceed the table's row limit");
 #ifndef ACS_HASH_PROWMAX
 #define ACS_HASH_PROWMAX 2048
 #endif

@@ -208,11 +208,11 @@ __global__ void k_block_bounds(const int32_t* __restrict__ arp, const int32_t* _
       if (hok) atomicAdd(&s_cand, 1);
       products[b] = sum;
       if (est) {
-        // POOL_BOUND (reading R40): a candidate's accumulator output is at most HASH_UMAX
+        // POOL_BOUND (reading R40): a candidate's accumulator output is at most HASH_UBOUND
         // columns per row (k_hash) or fewer (k_rows); its rows lie in [brs[b], brs[b+1]]
         const int64_t last = b + 1 < nblocks ? (int64_t)brs[b + 1] : rows_a - 1;
         const int64_t nr = last - brs[b] + 1;
-        est[b] = hok ? min(sum, nr * (int64_t)HASH_UMAX) : sum;
+        est[b] = hok ? min(sum, nr * (int64_t)HASH_UBOUND) : sum;
       }
       // the accumulators (R31, R33) emit up to one chunk per warp
       slots[b] = sum > 0 ? max((sum + (CAP - KEEP) - 1) / (CAP - KEEP), (int64_t)ACC_MAX_WARPS) +

@@ -862,7 +862,7 @@ void acspgemm_options_default(acspgemm_options* opt) {
   opt->collect_stage_times = 0;
   opt->num_segments = DEFAULT_SEGMENTS;
   opt->strategy = ACSPGEMM_STRATEGY_ADAPTIVE;
-  opt->pool_mode = ACSPGEMM_POOL_EXACT;
+  opt->pool_mode = ACSPGEMM_POOL_BOUND;
 }
 
 acspgemm_status acspgemm_plan_create(acspgemm_plan* plan, const acspgemm_options* opt) {

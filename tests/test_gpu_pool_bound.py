@@ -69,19 +69,19 @@ def overlapping_rows(n_rows=300, per_row=40, step=8, blen=32, seed=5):
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
 def test_bound_pool_same_bytes_stencil(dt, cuda_available):
     A = poisson3d_27pt(24)
-    ce, ie, *_ = run(A, A, dt)
+    ce, ie, *_ = run(A, A, dt, pool_mode="exact")
     cb, ib, *_ = run(A, A, dt, pool_mode="bound")
     assert digest(ce) == digest(cb)
     check_oracle(cb, A, A, dt)
     assert ie["pool_mode"] == 0 and ib["pool_mode"] == 1
-    assert ib["pool_bytes"] < 0.6 * ie["pool_bytes"]          # 27 x 27 products vs <= 256 per row
+    assert ib["pool_bytes"] < 0.6 * ie["pool_bytes"]          # 27 x 27 products vs <= 192 per row
     assert ib["ndeferred_blocks"] == 0 and ib["nhash_blocks"] == ie["nhash_blocks"] > 0
 
 
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
 def test_bound_pool_deferred_blocks(dt, cuda_available):
     A, B = overlapping_rows()
-    ce, ie, *_ = run(A, B, dt)
+    ce, ie, *_ = run(A, B, dt, pool_mode="exact")
     cb, ib, *_ = run(A, B, dt, pool_mode="bound")
     assert ib["ndeferred_blocks"] > 0                         # candidates that ended in AC-ESC
     assert digest(ce) == digest(cb)
@@ -102,7 +102,7 @@ def test_bound_pool_mixed_and_replay(cuda_available):
         return from_coo(X.rows + Y.rows, X.cols + Y.cols, rows, cols, vals)
     A = bdiag(A1, P)
     B = bdiag(B1, P)
-    ce, ie, *_ = run(A, B, np.float64)
+    ce, ie, *_ = run(A, B, np.float64, pool_mode="exact")
     cb, ib, plan, dA, dB, C = run(A, B, np.float64, pool_mode="bound")
     assert ib["ndeferred_blocks"] > 0 and ib["nhash_blocks"] > 0
     assert digest(ce) == digest(cb)
@@ -118,7 +118,7 @@ def test_bound_pool_mixed_and_replay(cuda_available):
     with torch.cuda.stream(s):
         plan.numeric_update(dA2, dB2, C, s)
     s.synchronize()
-    ref, *_ = run(A2, B2, np.float64)
+    ref, *_ = run(A2, B2, np.float64, pool_mode="exact")
     assert digest(C.to_numpy()) == digest(ref)
 
 
@@ -127,19 +127,19 @@ def test_auto_pool_under_limit(cuda_available):
     multiply succeeds in the bounded pool with the exact pool's bytes; EXACT fails."""
     p = pkg()
     A = poisson3d_27pt(20)
-    ce, ie, *_ = run(A, A, np.float64)
+    ce, ie, *_ = run(A, A, np.float64, pool_mode="exact")
     limit = int(0.5 * ie["pool_bytes"])
     ca, ia, *_ = run(A, A, np.float64, pool_mode="auto", pool_limit_bytes=limit)
     assert ia["pool_mode"] == 1 and digest(ca) == digest(ce)
     ca2, ia2, *_ = run(A, A, np.float64, pool_mode="auto")      # no limit: exact
     assert ia2["pool_mode"] == 0 and digest(ca2) == digest(ce)
     with pytest.raises(p.AcspgemmError) as ei:
-        run(A, A, np.float64, pool_limit_bytes=limit)
+        run(A, A, np.float64, pool_mode="exact", pool_limit_bytes=limit)
     assert ei.value.status == 4                                  # OUT_OF_MEMORY
 
 
 def test_bound_pool_esc_strategy_is_exact(cuda_available):
     A = random_csr(400, 400, 0.02, seed=4)
-    ce, ie, *_ = run(A, A, np.float64, strategy="esc")
+    ce, ie, *_ = run(A, A, np.float64, strategy="esc", pool_mode="exact")
     cb, ib, *_ = run(A, A, np.float64, strategy="esc", pool_mode="bound")
     assert ib["pool_mode"] == 0 and digest(ce) == digest(cb)
