@@ -60,8 +60,12 @@ __global__ void __launch_bounds__(32 * COPY_WARPS) k_copy(CopyArgs a) {
     if (i >= a.nshared) return;
     const SharedRow sh = a.shared[i];
     const int64_t dst = a.row_ptr[sh.row];
-    warp_copy<T>(a.merge_col + sh.merge_off, reinterpret_cast<const T*>(a.merge_val) + sh.merge_off,
-                 a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, sh.merged, lane);
+    if (sh.merge_off >= 0)
+      warp_copy<T>(a.merge_col + sh.merge_off, reinterpret_cast<const T*>(a.merge_val) + sh.merge_off,
+                   a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, sh.merged, lane);
+    else                                 // merged in place in the chunk pool (merge.cu)
+      warp_copy<T>(a.pool_col - sh.merge_off - 1, reinterpret_cast<const T*>(a.pool_val) - sh.merge_off - 1,
+                   a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, sh.merged, lane);
   }
 }
 

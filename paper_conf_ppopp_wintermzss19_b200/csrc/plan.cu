@@ -339,7 +339,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   // scal words: 0 products, 1 slots, 2 nblocks, 3 ncand / total chunks, 4 max block
   // products / shared rows, 5 bounded pool / chunk elements, 6 hash blocks, 7 dict
   // blocks, 8..14 merge class counts, 15 k_rows blocks, 16 nnz(C), 17-18 deferred blocks
-  // and their products, 20 nblocks (int32), 21 k_rows list, 23-25 dense slices, 26 k_rows
+  // and their products, 20 nblocks (int32), 21 k_rows list, 22 in-place merged elements,
+  // 23-25 dense slices, 26 k_rows
   // batches, 27 k_hash blocks, 28-31
   // AC-ESC lists.  The counters are zeroed by k_segments, the
   // first kernel (with err), and k_glb zeroes the per-row counters: no memset launches.
@@ -560,7 +561,8 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
   launch_find_shared(ms, L, scal + 4, st);
   tl_launches += 1 + (slots > 0 ? 7 : 0);
   ACS_CUDA(cudaGetLastError());
-  if ((s = sync_read(p, scal + 2, 14, st)) != ACSPGEMM_OK) return s;
+  if ((s = sync_read(p, scal + 2, 21, st)) != ACSPGEMM_OK) return s;
+  const int64_t inplace_total = p->h_scal[20];   // scal + 22: elements of rows merged in place
   p->info.nrow_blocks = p->h_scal[13];
   p->info.nhash_blocks = p->h_scal[4];
   p->info.ndict_blocks = p->h_scal[5];
@@ -588,7 +590,7 @@ acspgemm_status symbolic_impl(acspgemm_plan p, const acspgemm_csr_in* A, const a
     // Multi-Merge packing needs the multi totals: scan them over the multi list
     if (nmulti > 0) {
       // upper bound of groups from merge_total (multi totals <= merge_total)
-      int64_t gmax = 2 * ((merge_total + CAP - 1) / CAP) + 2;
+      int64_t gmax = 2 * ((merge_total + inplace_total + CAP - 1) / CAP) + 2;
       ACS_ENSURE(p->gstart, sizeof(int32_t) * 2 * (gmax + 1));
       L.group_start = ptr<int32_t>(p->gstart);
       launch_multi_groups(L, nmulti, gmax, st);
