@@ -109,8 +109,8 @@ struct SharedRow {
   int32_t first_chunk;    // dense global chunk index of the first chunk holding the row
   int32_t nchunks;
   int32_t total;          // sum of the row's element counts over its chunks (pre-merge)
-  int64_t merge_off;      // where the merged row goes in the merge pool; < 0: merged in place in
-                          // the chunk pool at -merge_off - 1 (its two pieces touch there)
+  int64_t merge_off;      // where the merged row goes in the merge pool; < 0: a two-chunk row
+                          // merged in place over its pieces (first piece's room, then the second's)
   int32_t merged;         // merged element count (written by the merge kernels)
   int32_t kind;           // 0 multi (block), 1 path, 2 search, 3 multi (warp pair), 4 dense slices
 };

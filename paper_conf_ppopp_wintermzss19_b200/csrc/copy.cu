@@ -63,9 +63,16 @@ __global__ void __launch_bounds__(32 * COPY_WARPS) k_copy(CopyArgs a) {
     if (sh.merge_off >= 0)
       warp_copy<T>(a.merge_col + sh.merge_off, reinterpret_cast<const T*>(a.merge_val) + sh.merge_off,
                    a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, sh.merged, lane);
-    else                                 // merged in place in the chunk pool (merge.cu)
-      warp_copy<T>(a.pool_col - sh.merge_off - 1, reinterpret_cast<const T*>(a.pool_val) - sh.merge_off - 1,
-                   a.c_col + dst, reinterpret_cast<T*>(a.c_val) + dst, sh.merged, lane);
+    else {                               // merged in place in the chunk pool (merge.cu): the first
+      const ChunkDesc d0 = a.dense[sh.first_chunk];              // piece's room, then the second's
+      const int64_t b0 = d0.data_off + d0.count - d0.last_count;
+      const int64_t b1 = a.dense[sh.first_chunk + 1].data_off;
+      const int n0 = min(sh.merged, d0.last_count);
+      const T* pv = reinterpret_cast<const T*>(a.pool_val);
+      T* cv = reinterpret_cast<T*>(a.c_val);
+      warp_copy<T>(a.pool_col + b0, pv + b0, a.c_col + dst, cv + dst, n0, lane);
+      warp_copy<T>(a.pool_col + b1, pv + b1, a.c_col + dst + n0, cv + dst + n0, sh.merged - n0, lane);
+    }
   }
 }
 
