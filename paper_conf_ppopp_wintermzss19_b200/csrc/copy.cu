@@ -17,7 +17,10 @@ namespace acs {
 template <typename T>
 __device__ __forceinline__ void warp_copy(const int32_t* __restrict__ scol, const T* __restrict__ sval,
                                           int32_t* __restrict__ dcol, T* __restrict__ dval, int n, int lane) {
-  constexpr int U = 8;
+#ifndef ACS_COPY_U
+#define ACS_COPY_U 8
+#endif
+  constexpr int U = ACS_COPY_U;
   int i = lane;
   for (; i + 32 * (U - 1) < n; i += 32 * U) {
     int32_t c[U];
@@ -39,7 +42,10 @@ __device__ __forceinline__ void warp_copy(const int32_t* __restrict__ scol, cons
   }
 }
 
-constexpr int COPY_WARPS = 8;
+#ifndef ACS_COPY_WARPS
+#define ACS_COPY_WARPS 8
+#endif
+constexpr int COPY_WARPS = ACS_COPY_WARPS;
 
 template <typename T>
 __global__ void __launch_bounds__(32 * COPY_WARPS) k_copy(CopyArgs a) {
