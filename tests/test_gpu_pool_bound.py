@@ -88,6 +88,20 @@ def test_bound_pool_deferred_blocks(dt, cuda_available):
     check_oracle(cb, A, B, dt)
 
 
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_bound_pool_row_cap(dt, cuda_available):
+    """Rows of 8*23 + 32 = 216 distinct columns: within the hash table's 256 (EXACT: k_hash
+    takes them) but over POOL_BOUND's cap of 192 per row (HASH_UBOUND), so in the bounded
+    pool k_hash gives the blocks up and they are deferred to AC-ESC -- the same bytes."""
+    A, B = overlapping_rows(n_rows=300, per_row=24, seed=11)
+    ce, ie, *_ = run(A, B, dt, pool_mode="exact")
+    cb, ib, *_ = run(A, B, dt, pool_mode="bound")
+    assert ie["nhash_blocks"] > 0 and ie["ndeferred_blocks"] == 0
+    assert ib["nhash_blocks"] < ie["nhash_blocks"] and ib["ndeferred_blocks"] > 0
+    assert digest(ce) == digest(cb)
+    check_oracle(cb, A, B, dt)
+
+
 def test_bound_pool_mixed_and_replay(cuda_available):
     """Deferred blocks next to hash blocks and short-row blocks in one multiply, then a
     graph replay (numeric_update) with new values: the same bytes as the exact pool."""
