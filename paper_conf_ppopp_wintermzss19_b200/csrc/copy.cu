@@ -8,6 +8,7 @@
 // B200: one warp per chunk (chunks average a few hundred elements), streaming
 // (evict-first) loads and stores since neither side is re-read.
 #include <algorithm>
+#include <climits>
 #include "kernels.cuh"
 
 namespace acs {
@@ -88,6 +89,31 @@ void launch_copy(const CopyArgs& a, bool f64, cudaStream_t st) {
   const unsigned grid = (unsigned)((items + COPY_WARPS - 1) / COPY_WARPS);
   if (f64) k_copy<double><<<grid, 32 * COPY_WARPS, 0, st>>>(a);
   else k_copy<float><<<grid, 32 * COPY_WARPS, 0, st>>>(a);
+}
+
+// min / max of col[0, n) into out[0] / out[1] (set to INT_MAX-ish / 0 first): the B rows a
+// row piece of A reaches (acspgemm_multiply_host's input pipeline).
+__global__ void k_col_range(const int32_t* __restrict__ col, int64_t n, int32_t* __restrict__ out) {
+  int mn = INT_MAX, mx = INT_MIN;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int c = col[i];
+    mn = min(mn, c);
+    mx = max(mx, c);
+  }
+  mn = __reduce_min_sync(0xffffffffu, mn);
+  mx = __reduce_max_sync(0xffffffffu, mx);
+  if ((threadIdx.x & 31) == 0) {
+    atomicMin(&out[0], mn);
+    atomicMax(&out[1], mx);
+  }
+}
+
+void launch_col_range(const int32_t* col, int64_t n, int32_t* out, cudaStream_t st) {
+  cudaMemsetAsync(out, 0x7F, sizeof(int32_t), st);
+  cudaMemsetAsync(out + 1, 0, sizeof(int32_t), st);
+  if (n <= 0) return;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 148 * 4);
+  k_col_range<<<grid, 256, 0, st>>>(col, n, out);
 }
 
 // Small read-backs go to mapped host memory through the SM (a copy-engine transfer would

@@ -209,6 +209,8 @@ void launch_rowptr_out(int32_t* dst, const int64_t* src, int64_t n, int32_t off,
 void launch_rowptr_out(int64_t* dst, const int64_t* src, int64_t n, int64_t off, cudaStream_t st);
 // dst[i] = src[i] + off (row pointers of a row piece placed after earlier pieces)
 void launch_copy_offset(int32_t* dst, const int32_t* src, int64_t n, int32_t off, cudaStream_t st);
+// out[0] = min, out[1] = max of col[0, n) (n = 0: out = {0x7F7F7F7F, 0})
+void launch_col_range(const int32_t* col, int64_t n, int32_t* out, cudaStream_t st);
 // nbytes (multiple of 4, <= 4096) from device memory to mapped host memory, by a kernel
 void launch_read_back(const void* src, void* mapped_dst, int nbytes, cudaStream_t st);
 // two read-backs in one launch

@@ -86,6 +86,9 @@ struct acspgemm_plan_s {
   DevBuf hp_a[3], hp_b[3], hp_c[2][3];
   cudaStream_t hp_cs = nullptr;
   cudaEvent_t hp_ready = nullptr, hp_copied[2] = {nullptr, nullptr};
+  cudaStream_t hp_in = nullptr;             // input copies (multiply_host), piece by piece
+  cudaEvent_t hp_start = nullptr, hp_inev[MAX_SEGMENTS + 1] = {};   // [S]: B when it is not A
+  DevBuf hp_rng;                            // a piece's column range
   int64_t* h_scal = nullptr;     // pinned read-back buffer
   cudaEvent_t ev[NSTAGE_EV];
   bool ev_ok = false;
@@ -839,6 +842,7 @@ struct HostPipeGuard {
   }
   ~HostPipeGuard() {
     if (plan->hp_cs) cudaStreamSynchronize(plan->hp_cs);
+    if (plan->hp_in) cudaStreamSynchronize(plan->hp_in);
     cudaStreamSynchronize(st);
     plan->nseg_explicit = saved_nseg;
     for (int i = 0; i <= MAX_SEGMENTS; ++i) plan->seg_rows_explicit[i] = saved_rows[i];
@@ -917,6 +921,10 @@ void acspgemm_plan_destroy(acspgemm_plan p) {
     free_buf(p->hp_c[1][i]);
   }
   if (p->hp_cs) cudaStreamDestroy(p->hp_cs);
+  if (p->hp_in) cudaStreamDestroy(p->hp_in);
+  if (p->hp_start) cudaEventDestroy(p->hp_start);
+  for (cudaEvent_t e : p->hp_inev) if (e) cudaEventDestroy(e);
+  free_buf(p->hp_rng);
   if (p->hp_ready) cudaEventDestroy(p->hp_ready);
   for (cudaEvent_t e : p->hp_copied) if (e) cudaEventDestroy(e);
   if (p->h_scal) cudaFreeHost(p->h_scal);
@@ -1188,30 +1196,35 @@ acspgemm_status acspgemm_multiply_host(acspgemm_plan p, const acspgemm_csr_in* A
   if (!p->hp_ready) ACS_CUDA(cudaEventCreateWithFlags(&p->hp_ready, cudaEventDisableTiming));
   for (cudaEvent_t& e : p->hp_copied)
     if (!e) ACS_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-  // inputs host -> device into plan memory (B once when it is A)
+  // inputs host -> device into plan memory (B once when it is A): the row pointers first
+  // (the segments need them), then the columns and values on an input stream, B whole
+  // (when it is not A) and A piece by piece, so piece g's multiply overlaps the copies of
+  // the pieces after it
+  if (!p->hp_in) ACS_CUDA(cudaStreamCreateWithFlags(&p->hp_in, cudaStreamNonBlocking));
+  if (!p->hp_start) ACS_CUDA(cudaEventCreateWithFlags(&p->hp_start, cudaEventDisableTiming));
+  for (cudaEvent_t& e : p->hp_inev)
+    if (!e) ACS_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
   const bool same = B->row_ptr == A->row_ptr && B->col_idx == A->col_idx && B->val == A->val &&
                     B->rows == A->rows && B->nnz == A->nnz;
   const acspgemm_csr_in* M[2] = {A, B};
   DevBuf* Dm[2] = {p->hp_a, p->hp_b};
   acspgemm_csr_in D[2];
+  int64_t hbase[2] = {0, 0};
   for (int m = 0; m < (same ? 1 : 2); ++m) {
     const acspgemm_csr_in* H = M[m];
     DevBuf* d = Dm[m];
     const int64_t base = H->rows > 0 ? H->row_ptr[0] : 0;
+    hbase[m] = base;
     ACS_ENSURE(d[0], sizeof(int32_t) * (H->rows + 1));
     ACS_ENSURE(d[1], sizeof(int32_t) * H->nnz);
     ACS_ENSURE(d[2], vb * H->nnz);
     ACS_CUDA(cudaMemcpyAsync(d[0].p, H->row_ptr, sizeof(int32_t) * (H->rows + 1), cudaMemcpyHostToDevice, st));
-    if (H->nnz > 0) {
-      ACS_CUDA(cudaMemcpyAsync(d[1].p, H->col_idx + base, sizeof(int32_t) * H->nnz, cudaMemcpyHostToDevice, st));
-      ACS_CUDA(cudaMemcpyAsync(d[2].p, static_cast<const char*>(H->val) + vb * base, vb * H->nnz,
-                               cudaMemcpyHostToDevice, st));
-    }
     // device view: row_ptr values index col / val directly (base shifted away)
     D[m] = acspgemm_csr_in{H->rows, H->cols, H->nnz, ptr<const int32_t>(d[0]), ptr<const int32_t>(d[1]) - base,
                            static_cast<const char*>(d[2].p) - vb * base};
   }
   if (same) D[1] = D[0];
+  hbase[1] = same ? hbase[0] : hbase[1];
   // canonical segments of the whole A (plan memory, one read-back), grouped into pieces
   int64_t seg[MAX_SEGMENTS + 1];
   {
@@ -1224,11 +1237,56 @@ acspgemm_status acspgemm_multiply_host(acspgemm_plan p, const acspgemm_csr_in* A
     ACS_CUDA(cudaMemcpyAsync(seg, sd, sizeof(int64_t) * (S + 1), cudaMemcpyDeviceToHost, st));
     ACS_CUDA(cudaStreamSynchronize(st));
   }
+  auto piece_rows = [&](int g, int64_t& r0, int64_t& r1) {
+    r0 = seg[(int)((int64_t)g * S / npieces)];
+    r1 = seg[(int)((int64_t)(g + 1) * S / npieces)];
+  };
+  ACS_CUDA(cudaEventRecord(p->hp_start, st));            // the input buffers are free from here
+  ACS_CUDA(cudaStreamWaitEvent(p->hp_in, p->hp_start, 0));
+  auto copy_nz = [&](int m, int64_t z0, int64_t z1) -> acspgemm_status {   // entries [z0, z1) of M[m]
+    if (z1 <= z0) return ACSPGEMM_OK;
+    const acspgemm_csr_in* H = M[m];
+    const int64_t o = z0 - hbase[m];
+    ACS_CUDA(cudaMemcpyAsync(ptr<int32_t>(Dm[m][1]) + o, H->col_idx + z0, sizeof(int32_t) * (z1 - z0),
+                             cudaMemcpyHostToDevice, p->hp_in));
+    ACS_CUDA(cudaMemcpyAsync(static_cast<char*>(Dm[m][2].p) + vb * o, static_cast<const char*>(H->val) + vb * z0,
+                             vb * (z1 - z0), cudaMemcpyHostToDevice, p->hp_in));
+    return ACSPGEMM_OK;
+  };
+  if (!same) {
+    if ((s = copy_nz(1, hbase[1], hbase[1] + B->nnz)) != ACSPGEMM_OK) return s;
+    ACS_CUDA(cudaEventRecord(p->hp_inev[S], p->hp_in));
+  }
+  for (int g = 0; g < npieces; ++g) {
+    int64_t r0, r1;
+    piece_rows(g, r0, r1);
+    if ((s = copy_nz(0, A->row_ptr[r0], A->row_ptr[r1])) != ACSPGEMM_OK) return s;
+    ACS_CUDA(cudaEventRecord(p->hp_inev[g], p->hp_in));
+  }
+  ACS_ENSURE(p->hp_rng, 2 * sizeof(int32_t));
   int64_t off = 0;
   bool overflow = false;
   for (int g = 0; g < npieces; ++g) {
     const int s0 = (int)((int64_t)g * S / npieces), s1 = (int)((int64_t)(g + 1) * S / npieces);
     const int64_t r0 = seg[s0], r1 = seg[s1];
+    ACS_CUDA(cudaStreamWaitEvent(st, p->hp_inev[g], 0));     // the piece's own rows of A
+    if (!same) {
+      ACS_CUDA(cudaStreamWaitEvent(st, p->hp_inev[S], 0));
+    } else if (A->row_ptr[r1] > A->row_ptr[r0]) {
+      // B is A: the rows of A this piece reaches, from its entries' column range (one
+      // read-back); the pieces holding them must have arrived
+      launch_col_range(D[0].col_idx + A->row_ptr[r0], (int64_t)A->row_ptr[r1] - A->row_ptr[r0], ptr<int32_t>(p->hp_rng), st);
+      launch_read_back(p->hp_rng.p, p->h_scal, 2 * sizeof(int32_t), st);
+      tl_launches += 2;
+      ACS_CUDA(cudaStreamSynchronize(st));
+      const int32_t* rng = reinterpret_cast<const int32_t*>(p->h_scal);
+      const int64_t z0 = A->row_ptr[rng[0]], z1 = A->row_ptr[(int64_t)rng[1] + 1];
+      for (int c = 0; c < npieces; ++c) {
+        int64_t q0, q1;
+        piece_rows(c, q0, q1);
+        if (c != g && A->row_ptr[q0] < z1 && A->row_ptr[q1] > z0) ACS_CUDA(cudaStreamWaitEvent(st, p->hp_inev[c], 0));
+      }
+    }
     p->nseg_explicit = s1 - s0;
     for (int i = 0; i <= s1 - s0; ++i) p->seg_rows_explicit[i] = seg[s0 + i] - r0;
     const acspgemm_csr_in V{r1 - r0, A->cols, (int64_t)A->row_ptr[r1] - A->row_ptr[r0], D[0].row_ptr + r0,

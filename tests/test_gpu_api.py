@@ -208,6 +208,21 @@ def test_multiply_host_pieces_bit_identical(pieces, cuda_available):
     assert (np.abs(val.numpy() - ref.val) <= 1e-12 * ref.absval).all()
 
 
+@pytest.mark.parametrize("pieces", [2, 8])
+def test_multiply_host_banded_inputs_in_pieces(pieces, cuda_available):
+    """B is A and banded: a piece waits only for the input pieces holding the rows its
+    entries reach (their column range, read back per piece), the later pieces' copies
+    still in flight -- C equals the device multiply byte for byte."""
+    from synth import poisson3d_27pt
+    p = pkg()
+    A = poisson3d_27pt(24)
+    full = p.multiply(dev(A), dev(A))
+    frp, fcol, fval = full.to_numpy()
+    rp, col, val = p.multiply_host(A, A, pieces=pieces)
+    assert (rp.numpy() == frp).all() and (col.numpy() == fcol).all()
+    assert val.numpy().tobytes() == fval.tobytes()
+
+
 def test_multiply_host_rectangular_capacity(cuda_available):
     """B distinct from A (copied separately), numpy buffers, capacity overflow reports nnz."""
     p = pkg()
