@@ -49,7 +49,7 @@ __device__ __forceinline__ void warp_copy(const int32_t* __restrict__ scol, cons
 constexpr int COPY_WARPS = ACS_COPY_WARPS;
 
 template <typename T>
-__global__ void __launch_bounds__(32 * COPY_WARPS) k_copy(CopyArgs a) {
+__global__ void __launch_bounds__(32 * COPY_WARPS, 5) k_copy(CopyArgs a) {   // 5 CTAs per SM: <= 48 registers
   const int64_t x = (int64_t)blockIdx.x * COPY_WARPS + (threadIdx.x >> 5);
   const int lane = threadIdx.x & 31;
   if (x < a.max_chunks) {

@@ -216,7 +216,7 @@ __device__ __forceinline__ void rows_block(RowsSmem<T>& S, const EscArgs& a, con
 constexpr int ROWS_BATCH = 32;
 
 template <typename T>
-__global__ void __launch_bounds__(THREADS) k_rows(EscArgs a) {
+__global__ void __launch_bounds__(THREADS, 8) k_rows(EscArgs a) {   // 8 CTAs per SM (26 KB shared memory each)
   extern __shared__ __align__(16) unsigned char smem_raw[];
   RowsSmem<T>& S = *reinterpret_cast<RowsSmem<T>*>(smem_raw);
   const int tid = threadIdx.x;
