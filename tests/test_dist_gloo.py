@@ -1,5 +1,5 @@
 """Multi-process host logic of the row-segment multi-GPU driver on CPU (gloo,
-world_size 2 and 4): canonical segments, per-rank ownership, (rows, nnz) all-gather
+world_size 2, 4 and 8 -- one canonical segment per rank at 8): canonical segments, per-rank ownership, (rows, nnz) all-gather
 offsets, CSR broadcast and concatenation.  The per-rank multiply is the oracle here
 (a CPU stand-in injected by the test; the product path itself has no CPU fallback)."""
 import os
@@ -60,7 +60,7 @@ def _worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("world", [2, 4, 8])
 def test_dist_multiply_gloo(world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
